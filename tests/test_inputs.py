@@ -1,0 +1,87 @@
+"""The seeded input generators (micco_inputs): the numpy generator agrees bit for
+bit with the C header both native sides include, and the graph recipes have
+the structure SURVEY.md §8(d) states."""
+import collections
+
+import numpy as np
+import pytest
+
+import oracle
+from micco_inputs import workloads, synth_node
+from micco_inputs.gen import MODE_INT3, MODE_UNIFORM, node_scale
+
+
+@pytest.mark.parametrize("mode", [MODE_UNIFORM, MODE_INT3])
+@pytest.mark.parametrize("rank,N,Lt", [(2, 5, 3), (3, 4, 2), (2, 32, 8)])
+def test_numpy_generator_matches_c_header(mode, rank, N, Lt):
+    wl = workloads.Workload("t", Lt, 12345, mode, [workloads.NodeSpec(rank, N, 77)], [])
+    tb = oracle.NodeTable(wl)
+    a = tb.tensor(0)
+    b = synth_node(12345, 77, rank, N, Lt, mode)
+    assert a.shape == b.shape
+    assert np.array_equal(a.view(np.uint64), b.view(np.uint64))
+
+
+def test_generator_ranges():
+    x = synth_node(1, 2, 2, 64, 4, MODE_UNIFORM)
+    s = node_scale(2, 64)
+    assert np.all(np.abs(x.real) <= s) and np.all(np.abs(x.imag) <= s)
+    assert abs(np.mean(x.real)) < 0.05 * s
+    y = synth_node(1, 2, 3, 8, 4, MODE_INT3)
+    assert set(np.unique(y.real)) == {-1.0, 0.0, 1.0}
+    # different keys / seeds give different streams
+    assert not np.array_equal(synth_node(1, 3, 2, 8, 2), synth_node(1, 2, 2, 8, 2))
+    assert not np.array_equal(synth_node(2, 2, 2, 8, 2), synth_node(1, 2, 2, 8, 2))
+
+
+def _valid_matching(wl, G):
+    legs = collections.Counter()
+    for (u, p, v, q) in G.edges:
+        assert 0 <= p < wl.nodes[G.inst[u]].rank and 0 <= q < wl.nodes[G.inst[v]].rank
+        legs[(u, p)] += 1
+        legs[(v, q)] += 1
+    total = sum(wl.nodes[n].rank for n in G.inst)
+    assert len(legs) == total and all(c == 1 for c in legs.values())
+    if G.order is not None:
+        assert sorted(G.order) == list(range(len(G.edges)))
+
+
+def test_c1_structure():
+    wl = workloads.c1_two_meson()
+    assert len(wl.graphs) == 32 and wl.Lt == 8 and all(n.N == 32 and n.rank == 2 for n in wl.nodes)
+    sizes = collections.Counter(len(G.inst) for G in wl.graphs)
+    assert sizes == {2: 8, 3: 8, 4: 16}
+    for G in wl.graphs:
+        _valid_matching(wl, G)
+
+
+def test_c2_repetition_rate():
+    for rate in (0.1, 0.5, 0.9):
+        wl = workloads.c2_meson_set(n_graphs=2000, N=8, Lt=2, rate=rate)
+        slots = sum(len(G.inst) for G in wl.graphs)
+        repeated = 1.0 - len(wl.nodes) / slots
+        assert abs(repeated - rate) < 0.05, (rate, repeated)
+        for G in wl.graphs[:50]:
+            _valid_matching(wl, G)
+    g = workloads.c2_meson_set(n_graphs=2000, N=8, Lt=2, rate=0.5, dist="gaussian")
+    assert len(g.graphs) == 2000
+
+
+def test_c3_cycle_structure():
+    wl = workloads.c3_multi_meson(n_graphs=500, N=4, Lt=2)
+    for G in wl.graphs:
+        _valid_matching(wl, G)
+        # every edge joins a sink (0..2) and a source (3..5)
+        assert all((u < 3) != (v < 3) for (u, _, v, _) in G.edges)
+
+
+def test_c4_matchings():
+    m = workloads.two_baryon_matchings()
+    assert len(m) == 720
+    # k = legs S1 shares with R1: 72 disconnected (k = 0 or 3), 648 connected
+    ks = collections.Counter(sum(1 for s, r in mm if s < 3 and r < 3) for mm in m)
+    assert ks[0] + ks[3] == 72 and ks[1] + ks[2] == 648
+    wl = workloads.c4_two_baryon(n_combos=2, N=3, Lt=1, order="chain")
+    assert len(wl.graphs) == 1440
+    for G in wl.graphs[:100]:
+        _valid_matching(wl, G)
