@@ -1,0 +1,196 @@
+// core.h — internal data model of the MICCO engine (host side).
+//
+// Tensors: hadron nodes (inputs) and the intermediates produced by pairwise
+// hadron contractions (L17-19, L60) share one id space.  A Task is one unique pairwise
+// contraction after hash-consing (shared reduction paths, L23).  Graphs keep the scalar
+// tensors of their connected components and their coefficient.
+#pragma once
+
+#include <cstdint>
+#include <cstring>
+#include <memory>
+#include <string>
+#include <unordered_map>
+#include <vector>
+
+#include "micco.h"
+
+namespace micco {
+
+constexpr int kMaxRank = 4;  // intermediate rank cap
+
+struct Error {
+  micco_status code;
+  std::string msg;
+};
+
+[[noreturn]] void fail(micco_status code, const std::string &msg);
+
+struct NodeRec {
+  int32_t rank = 0, N = 0;
+  int64_t slice_elems = 0;  // N^rank complex elements per time slice
+  double *host = nullptr;   // 2 * Lt * slice_elems doubles, interleaved, t slowest
+  uint64_t hash = 0;
+  int32_t tensor = -1;
+};
+
+enum TaskKind : int8_t { TASK_GEMM = 0, TASK_DOT = 1, TASK_TRACE = 2 };
+
+struct TensorRec {
+  int32_t rank = 0;                  // 0 = per-slice scalar
+  int32_t dim[kMaxRank] = {0, 0, 0, 0};
+  int64_t slice_elems = 1;
+  int32_t node = -1;                 // >= 0: an input hadron node
+  int32_t task = -1;                 // >= 0: produced by this task
+  int32_t level = 0;                 // 0 for nodes, 1 + max(operand levels) for task outputs
+  int32_t scalar_slot = -1;          // rank 0: row of the scalar table
+  int64_t bytes(int32_t Lt) const { return slice_elems * (int64_t)Lt * 16; }
+};
+
+// One unique pairwise contraction.  out[legs] = Σ_k a[...] b[...] with the contracted leg
+// pairs (pa[i], pb[i]) sorted by pa; result legs = a's free legs in order, then b's
+// (SURVEY.md §8(c) #9).  TRACE: a is a meson, out = Σ_i a[i][i].
+struct TaskRec {
+  TaskKind kind = TASK_GEMM;
+  int32_t a = -1, b = -1;
+  int8_t c = 0;
+  int8_t pa[kMaxRank] = {0, 0, 0, 0}, pb[kMaxRank] = {0, 0, 0, 0};
+  int32_t out = -1;
+  int32_t level = 0;
+  double flops = 0;                  // 8 real flops per complex MAC, all Lt slices
+  int32_t uses = 0;                  // consumers (task operands + graph scalars)
+};
+
+struct TaskKey {
+  int32_t a, b;
+  int8_t c;
+  int8_t pa[kMaxRank], pb[kMaxRank];
+  bool operator==(const TaskKey &o) const {
+    return a == o.a && b == o.b && c == o.c && std::memcmp(pa, o.pa, sizeof pa) == 0 &&
+           std::memcmp(pb, o.pb, sizeof pb) == 0;
+  }
+};
+struct TaskKeyHash {
+  size_t operator()(const TaskKey &k) const {
+    uint64_t h = 1469598103934665603ULL;
+    auto mix = [&](uint64_t x) { h = (h ^ x) * 1099511628211ULL; };
+    mix((uint32_t)k.a); mix((uint32_t)k.b); mix((uint8_t)k.c);
+    for (int i = 0; i < kMaxRank; ++i) { mix((uint8_t)k.pa[i]); mix((uint8_t)k.pb[i]); }
+    return (size_t)h;
+  }
+};
+
+struct GraphRec {
+  double coef_re = 1, coef_im = 0;
+  int32_t comp_begin = 0, comp_end = 0;  // range in Context::graph_scalars
+  double flops_no_dedup = 0;
+};
+
+struct SynthKey {
+  uint64_t seed, key;
+  int32_t mode, rank, N;
+  double scale;
+  bool operator==(const SynthKey &o) const {
+    return seed == o.seed && key == o.key && mode == o.mode && rank == o.rank && N == o.N &&
+           std::memcmp(&scale, &o.scale, sizeof scale) == 0;
+  }
+};
+struct SynthKeyHash {
+  size_t operator()(const SynthKey &k) const {
+    uint64_t s;
+    std::memcpy(&s, &k.scale, 8);
+    return (size_t)((k.seed * 0x9E3779B97F4A7C15ULL) ^ (k.key * 0xC2B2AE3D27D4EB4FULL) ^
+                    ((uint64_t)k.mode << 7) ^ ((uint64_t)k.rank << 13) ^ ((uint64_t)k.N << 17) ^ s);
+  }
+};
+
+// Pinned host memory for node tensors and spills: 1 GiB chunks (cudaHostAlloc when a CUDA
+// device is present, else page-aligned malloc so the host-only paths work without a GPU).
+class HostArena {
+ public:
+  ~HostArena();
+  double *alloc(int64_t bytes);
+  bool pinned() const { return pinned_; }
+  void release_all();
+ private:
+  struct Chunk { char *base; int64_t size, used; bool pinned; };
+  std::vector<Chunk> chunks_;
+  std::vector<std::pair<char *, bool>> big_;
+  bool pinned_ = true;
+};
+
+class Executor;  // executor.cu
+
+struct Plan;     // planner.cpp
+
+struct Context {
+  micco_options opt{};
+  std::string last_error;
+  bool sticky = false;
+  int32_t Lt = -1;
+  HostArena arena;
+  std::vector<NodeRec> nodes;
+  std::unordered_multimap<uint64_t, int32_t> node_by_hash;
+  std::unordered_map<SynthKey, int32_t, SynthKeyHash> node_by_synth;
+  std::vector<TensorRec> tensors;
+  std::vector<TaskRec> tasks;
+  std::unordered_map<TaskKey, int32_t, TaskKeyHash> task_by_key;
+  std::vector<GraphRec> graphs;
+  std::vector<int32_t> graph_scalars;  // tensor ids (rank 0), grouped per graph
+  int64_t dedup_hits = 0;
+  int32_t n_scalar_slots = 0;
+  // results of the last execute
+  bool have_result = false;
+  std::vector<double> corr;        // 2 * Lt
+  std::vector<double> graph_vals;  // 2 * G * Lt, filled lazily
+  bool graph_vals_valid = false;
+  micco_stats stats{};
+  std::unique_ptr<Executor> exec;
+  uint8_t nccl_id[128] = {0};
+  bool have_nccl_id = false;
+  Context();
+  ~Context();
+};
+
+// builder.cpp
+int32_t add_node_tensor(Context &ctx, int32_t node);
+void build_graph(Context &ctx, int32_t n_inst, const int64_t *node_ids, int32_t n_edges,
+                 const micco_edge *edges, const int32_t *order, double cre, double cim);
+uint64_t content_hash(const double *data, int64_t n_doubles);
+
+// planner.cpp
+struct PlanOp {
+  enum Kind : uint8_t { H2D = 0, P2P = 1, SPILL = 2, FREE = 3, COMPUTE = 4, FLUSH = 5 };
+  Kind kind;
+  int32_t gpu;     // GPU that executes the op (P2P: destination)
+  int32_t src;     // P2P: source GPU
+  int32_t id;      // tensor (H2D/P2P/SPILL/FREE) or task (COMPUTE)
+};
+
+struct Plan {
+  int32_t n_gpus = 1;
+  int32_t reuse_bound[3] = {0, 0, 0};
+  std::vector<PlanOp> ops;
+  std::vector<int32_t> task_gpu;
+  std::vector<int64_t> gpu_peak_bytes;
+  int64_t bytes_h2d = 0, bytes_p2p = 0, bytes_d2h = 0, evictions = 0, cache_hits = 0;
+  int64_t n_stages = 0;
+  double flops = 0, max_over_mean_load = 1, predicted_s = 0;
+  std::vector<double> gpu_flops;
+};
+
+struct PlanInput {
+  int32_t n_gpus;
+  int32_t policy;
+  int32_t reuse_bound[3];
+  std::vector<int64_t> budget;                      // per GPU
+  int32_t window_graphs;
+  bool keep_inputs;
+  std::vector<std::vector<int32_t>> initial_nodes;  // per GPU: node tensors already resident
+  double peer_gbs, host_gbs, flops_per_s;           // cost model of the bound sweep
+};
+
+Plan make_plan(const Context &ctx, const PlanInput &in);
+Plan make_plan_auto(const Context &ctx, PlanInput in);  // sweeps reuse bounds when asked
+
+}  // namespace micco

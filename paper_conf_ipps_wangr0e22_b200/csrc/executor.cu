@@ -1,0 +1,718 @@
+// executor.cu — replays the planner's op list on 1..64 (logical) GPUs.
+//
+//  * one CUDA stream per logical GPU; logical GPU g runs on device g % device_count, so the
+//    multi-GPU scheduling / cache / P2P paths also run (as device-local copies) on one B200;
+//  * tensors live in stream-ordered pool allocations (cudaMallocAsync), interleaved complex;
+//  * H2D from the library's pinned node store, NVLink peer copies (cudaMemcpyPeerAsync) for
+//    replicas held by another GPU, D2H spills of sole copies under memory pressure
+//    (allocation and CPU↔GPU / GPU↔GPU movement are the memory
+//    operations the scheduler trades against load balance);
+//  * the tasks of one stage and GPU are batched into one grouped GEMM launch and one grouped
+//    dot launch (descriptors staged through a pinned ring);
+//  * rank-0 results land in a per-device scalar table [slot][t]; devices are combined by an
+//    exact sum (each slot is nonzero on one device only): NCCL all-reduce in multi-process
+//    mode, peer copies otherwise; then C(t) = Σ_g c_g Π_comp s_comp(t) on device 0.
+// Multi-process mode (one process per GPU): every rank replays the same plan, executes only
+// its own GPU's ops, and turns cross-GPU copies into matched ncclSend / ncclRecv.
+#include <cuda_runtime.h>
+#include <dlfcn.h>
+#include <nccl.h>
+
+#include <algorithm>
+#include <chrono>
+#include <cstring>
+#include <string>
+#include <unordered_map>
+
+#include "executor.h"
+#include "kernels.h"
+#include "layout.h"
+
+namespace micco {
+
+#define CK(x)                                                                                       \
+  do {                                                                                              \
+    cudaError_t e_ = (x);                                                                           \
+    if (e_ != cudaSuccess)                                                                          \
+      fail(MICCO_ERR_CUDA, std::string("CUDA error: ") + cudaGetErrorString(e_) + " at " #x);       \
+  } while (0)
+
+// ------------------------------------------------------------------ NCCL (dlopen)
+
+namespace {
+
+struct NcclApi {
+  bool ok = false;
+  std::string why;
+  ncclResult_t (*GetUniqueId)(ncclUniqueId *);
+  ncclResult_t (*CommInitRank)(ncclComm_t *, int, ncclUniqueId, int);
+  ncclResult_t (*CommInitAll)(ncclComm_t *, int, const int *);
+  ncclResult_t (*CommDestroy)(ncclComm_t);
+  ncclResult_t (*AllReduce)(const void *, void *, size_t, ncclDataType_t, ncclRedOp_t, ncclComm_t, cudaStream_t);
+  ncclResult_t (*Send)(const void *, size_t, ncclDataType_t, int, ncclComm_t, cudaStream_t);
+  ncclResult_t (*Recv)(void *, size_t, ncclDataType_t, int, ncclComm_t, cudaStream_t);
+  ncclResult_t (*GroupStart)();
+  ncclResult_t (*GroupEnd)();
+  const char *(*GetErrorString)(ncclResult_t);
+};
+
+NcclApi &nccl() {
+  static NcclApi api = [] {
+    NcclApi a;
+    void *h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_GLOBAL);
+    if (!h) h = dlopen("libnccl.so", RTLD_NOW | RTLD_GLOBAL);
+    if (!h) { a.why = "libnccl.so.2 not loadable"; return a; }
+#define LOAD(name) a.name = reinterpret_cast<decltype(a.name)>(dlsym(h, "nccl" #name)); if (!a.name) { a.why = "missing nccl" #name; return a; }
+    LOAD(GetUniqueId) LOAD(CommInitRank) LOAD(CommInitAll) LOAD(CommDestroy) LOAD(AllReduce)
+    LOAD(Send) LOAD(Recv) LOAD(GroupStart) LOAD(GroupEnd) LOAD(GetErrorString)
+#undef LOAD
+    a.ok = true;
+    return a;
+  }();
+  return api;
+}
+
+#define NK(x)                                                                                       \
+  do {                                                                                              \
+    ncclResult_t r_ = (x);                                                                          \
+    if (r_ != ncclSuccess) fail(MICCO_ERR_NCCL, std::string("NCCL error: ") + nccl().GetErrorString(r_)); \
+  } while (0)
+
+}  // namespace
+
+micco_status nccl_unique_id(uint8_t out[128]) {
+  NcclApi &a = nccl();
+  if (!a.ok) return MICCO_ERR_NCCL;
+  ncclUniqueId id;
+  if (a.GetUniqueId(&id) != ncclSuccess) return MICCO_ERR_NCCL;
+  std::memcpy(out, &id, 128);
+  return MICCO_OK;
+}
+
+// ------------------------------------------------------------------ executor state
+
+namespace {
+
+constexpr int kRingSlots = 64;
+constexpr size_t kSlotBytes = 256 * 1024;
+
+struct EventPool {
+  int dev = -1;
+  unsigned flags = cudaEventDisableTiming;
+  std::vector<cudaEvent_t> all;
+  size_t used = 0;
+  cudaEvent_t get() {
+    if (used == all.size()) {
+      cudaEvent_t e;
+      CK(cudaSetDevice(dev));
+      CK(cudaEventCreateWithFlags(&e, flags));
+      all.push_back(e);
+    }
+    return all[used++];
+  }
+  void reset() { used = 0; }
+  void destroy() {
+    if (dev >= 0) cudaSetDevice(dev);
+    for (auto e : all) cudaEventDestroy(e);
+    all.clear();
+    used = 0;
+  }
+};
+
+struct DevState {
+  int dev = -1;
+  double2 *scalars = nullptr;
+  size_t scalar_elems = 0;
+  EventPool sync_events, timing_events;
+  bool init = false;
+};
+
+struct Timed {
+  cudaEvent_t a, b;
+  int kind;  // 0 gemm, 1 dot, 2 copy
+  int dev;
+};
+
+struct LGpu {
+  int idx = 0, dev = 0;
+  bool local = true;
+  cudaStream_t st = nullptr;
+  std::vector<double2 *> ptr;                                  // tensor → replica
+  std::unordered_map<int32_t, std::vector<cudaEvent_t>> readers;  // peer reads to wait for before free
+  std::vector<GemmDesc> gemm;
+  std::vector<DotDesc> dot;
+  long long gemm_tiles = 0, dot_ctas = 0;
+  char *ring_h = nullptr, *ring_d = nullptr;
+  cudaEvent_t ring_ev[kRingSlots] = {};
+  bool ring_used[kRingSlots] = {};
+  int ring_next = 0;
+};
+
+}  // namespace
+
+struct Executor::Impl {
+  Context &c;
+  int ndev = 0;
+  int n = 0;  // logical GPUs
+  std::vector<LGpu> g;
+  std::vector<DevState> devs;
+  std::vector<Timed> timed;
+  std::unordered_map<int32_t, double *> spill_host;
+  std::unordered_map<int32_t, std::pair<int, cudaEvent_t>> spill_ev;
+  HostArena spill_arena;
+  ncclComm_t comm = nullptr;
+  std::vector<ncclComm_t> comms_all;  // single-process multi-device
+  std::vector<int64_t> budget_cache;
+  int budget_cache_n = 0;
+  int32_t chosen_bd[3] = {0, 0, 0};
+  int chosen_bd_n = 0;
+  // results on device 0
+  double2 *d_vals = nullptr;
+  size_t vals_elems = 0;
+  double2 *h_corr = nullptr;
+  int64_t launches = 0;
+  bool dist() const { return c.opt.dist_world > 0; }
+  int my_rank() const { return c.opt.dist_rank; }
+
+  explicit Impl(Context &ctx) : c(ctx) {}
+  ~Impl() { teardown(); }
+
+  void teardown() {
+    for (auto &l : g) free_lgpu(l, true);
+    g.clear();
+    n = 0;
+    for (auto &d : devs) {
+      if (d.dev < 0) continue;
+      cudaSetDevice(d.dev);
+      if (d.scalars) cudaFree(d.scalars);
+      d.scalars = nullptr;
+      d.sync_events.destroy();
+      d.timing_events.destroy();
+    }
+    if (d_vals) { cudaSetDevice(devs.empty() ? 0 : devs[0].dev); cudaFree(d_vals); d_vals = nullptr; }
+    if (h_corr) { cudaFreeHost(h_corr); h_corr = nullptr; }
+    if (comm && nccl().ok) nccl().CommDestroy(comm);
+    comm = nullptr;
+    for (auto cm : comms_all) if (cm && nccl().ok) nccl().CommDestroy(cm);
+    comms_all.clear();
+  }
+
+  void free_lgpu(LGpu &l, bool destroy_stream) {
+    if (!l.local || !l.st) return;
+    cudaSetDevice(l.dev);
+    for (auto &p : l.ptr)
+      if (p) { cudaFreeAsync(p, l.st); p = nullptr; }
+    cudaStreamSynchronize(l.st);
+    l.readers.clear();
+    if (destroy_stream) {
+      for (int i = 0; i < kRingSlots; ++i)
+        if (l.ring_ev[i]) cudaEventDestroy(l.ring_ev[i]);
+      if (l.ring_h) cudaFreeHost(l.ring_h);
+      if (l.ring_d) cudaFree(l.ring_d);
+      cudaStreamDestroy(l.st);
+      l.st = nullptr;
+    }
+  }
+
+  void setup(int n_gpus) {
+    CK(cudaGetDeviceCount(&ndev));
+    if (ndev < 1) fail(MICCO_ERR_CUDA, "no CUDA device (micco has no CPU fallback)");
+    if (n_gpus == n && !g.empty()) return;
+    teardown();
+    n = n_gpus;
+    devs.assign(ndev, DevState{});
+    for (int d = 0; d < ndev; ++d) {
+      devs[d].dev = d;
+      devs[d].sync_events.dev = d;
+      devs[d].timing_events.dev = d;
+      devs[d].timing_events.flags = cudaEventDefault;
+    }
+    g.assign(n, LGpu{});
+    for (int i = 0; i < n; ++i) {
+      LGpu &l = g[i];
+      l.idx = i;
+      l.dev = i % ndev;
+      l.local = !dist() || i == my_rank();
+      if (!l.local) continue;
+      CK(cudaSetDevice(l.dev));
+      if (!devs[l.dev].init) {
+        cudaMemPool_t pool;
+        CK(cudaDeviceGetDefaultMemPool(&pool, l.dev));
+        uint64_t thr = UINT64_MAX;
+        CK(cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr));
+        for (int p = 0; p < ndev; ++p) {  // NVLink peer access for P2P replicas
+          if (p == l.dev) continue;
+          int can = 0;
+          cudaDeviceCanAccessPeer(&can, l.dev, p);
+          if (can) {
+            cudaError_t e = cudaDeviceEnablePeerAccess(p, 0);
+            if (e != cudaSuccess && e != cudaErrorPeerAccessAlreadyEnabled) CK(e);
+            cudaGetLastError();
+          }
+        }
+        devs[l.dev].init = true;
+      }
+      CK(cudaStreamCreateWithFlags(&l.st, cudaStreamNonBlocking));
+      CK(cudaHostAlloc((void **)&l.ring_h, kRingSlots * kSlotBytes, cudaHostAllocPortable));
+      CK(cudaMalloc((void **)&l.ring_d, kRingSlots * kSlotBytes));
+      for (int s = 0; s < kRingSlots; ++s) CK(cudaEventCreateWithFlags(&l.ring_ev[s], cudaEventDisableTiming));
+    }
+    if (dist()) {
+      if (!c.have_nccl_id) fail(MICCO_ERR_STATE, "multi-process mode needs micco_set_nccl_id before execute");
+      if (!nccl().ok) fail(MICCO_ERR_NCCL, "NCCL unavailable: " + nccl().why);
+      ncclUniqueId id;
+      std::memcpy(&id, c.nccl_id, 128);
+      CK(cudaSetDevice(g[my_rank()].dev));
+      NK(nccl().CommInitRank(&comm, n, id, my_rank()));
+    }
+    budget_cache_n = 0;
+  }
+
+  std::vector<int64_t> budgets() {
+    if (budget_cache_n == n) return budget_cache;
+    std::vector<int64_t> b(n);
+    std::vector<int> per_dev(ndev, 0);
+    for (int i = 0; i < n; ++i) per_dev[g[i].dev]++;
+    for (int i = 0; i < n; ++i) {
+      if (c.opt.mem_budget_bytes > 0) { b[i] = c.opt.mem_budget_bytes; continue; }
+      size_t fr = 0, tot = 0;
+      if (g[i].local || !dist()) {
+        CK(cudaSetDevice(g[i].dev));
+        CK(cudaMemGetInfo(&fr, &tot));
+      } else {
+        // remote ranks: assume the same device model as ours (identical plan on every rank)
+        CK(cudaSetDevice(g[my_rank()].dev));
+        CK(cudaMemGetInfo(&fr, &tot));
+      }
+      int k = dist() ? 1 : per_dev[g[i].dev];
+      int64_t usable = (int64_t)(fr * 0.92) - (2LL << 30);
+      b[i] = std::max<int64_t>(usable / k, 1LL << 28);
+    }
+    if (dist()) {  // every rank must plan with identical budgets
+      int64_t mn = *std::min_element(b.begin(), b.end());
+      std::fill(b.begin(), b.end(), mn);
+    }
+    budget_cache = b;
+    budget_cache_n = n;
+    return b;
+  }
+
+  // ---------------------------------------------------------------- op replay
+
+  cudaEvent_t record(int gi) {
+    LGpu &l = g[gi];
+    cudaEvent_t e = devs[l.dev].sync_events.get();
+    CK(cudaSetDevice(l.dev));
+    CK(cudaEventRecord(e, l.st));
+    return e;
+  }
+
+  double2 *alloc(LGpu &l, int64_t bytes) {
+    void *p = nullptr;
+    CK(cudaMallocAsync(&p, (size_t)bytes, l.st));
+    return (double2 *)p;
+  }
+
+  int64_t bytes_of(int32_t x) const { return c.tensors[x].bytes(c.Lt); }
+
+  const double *host_src(int32_t x) const {
+    const TensorRec &t = c.tensors[x];
+    if (t.node >= 0) return c.nodes[t.node].host;
+    auto it = spill_host.find(x);
+    if (it == spill_host.end()) fail(MICCO_ERR_STATE, "executor: missing host copy");
+    return it->second;
+  }
+
+  char *ring_slot(LGpu &l, size_t bytes, int &slot) {
+    if (bytes > kSlotBytes) fail(MICCO_ERR_STATE, "descriptor batch too large");
+    slot = l.ring_next;
+    l.ring_next = (l.ring_next + 1) % kRingSlots;
+    if (l.ring_used[slot]) CK(cudaEventSynchronize(l.ring_ev[slot]));
+    l.ring_used[slot] = true;
+    return l.ring_h + (size_t)slot * kSlotBytes;
+  }
+
+  template <typename D, typename Launch>
+  void launch_batch(LGpu &l, std::vector<D> &v, int kind, Launch &&launch) {
+    if (v.empty()) return;
+    const size_t per = kSlotBytes / sizeof(D);
+    for (size_t i0 = 0; i0 < v.size(); i0 += per) {
+      size_t cnt = std::min(per, v.size() - i0);
+      int slot;
+      char *h = ring_slot(l, cnt * sizeof(D), slot);
+      std::memcpy(h, &v[i0], cnt * sizeof(D));
+      long long first = 0, total = 0;
+      D *hd = (D *)h;
+      launch(hd, (int)cnt, first, total);  // fixes offsets in the staged copy
+      char *dptr = l.ring_d + (size_t)slot * kSlotBytes;
+      CK(cudaMemcpyAsync(dptr, h, cnt * sizeof(D), cudaMemcpyHostToDevice, l.st));
+      CK(cudaEventRecord(l.ring_ev[slot], l.st));
+      Timed tm{devs[l.dev].timing_events.get(), devs[l.dev].timing_events.get(), kind, l.dev};
+      CK(cudaEventRecord(tm.a, l.st));
+      if (kind == 0) CK(launch_gemm_group((const GemmDesc *)dptr, (int)cnt, total, l.st));
+      else CK(launch_dot_group((const DotDesc *)dptr, (int)cnt, total, l.st));
+      CK(cudaEventRecord(tm.b, l.st));
+      timed.push_back(tm);
+      ++launches;
+    }
+    v.clear();
+  }
+
+  void flush(LGpu &l) {
+    CK(cudaSetDevice(l.dev));
+    launch_batch(l, l.gemm, 0, [](GemmDesc *d, int cnt, long long &first, long long &total) {
+      long long acc = 0;
+      for (int i = 0; i < cnt; ++i) {
+        long long tiles = (long long)d[i].Lt * d[i].Mo * d[i].No * d[i].tilesM * d[i].tilesN;
+        d[i].tile_begin = acc;
+        acc += tiles;
+      }
+      first = 0;
+      total = acc;
+    });
+    launch_batch(l, l.dot, 1, [](DotDesc *d, int cnt, long long &first, long long &total) {
+      long long acc = 0;
+      for (int i = 0; i < cnt; ++i) {
+        d[i].cta_begin = acc;
+        acc += d[i].Lt;
+      }
+      first = 0;
+      total = acc;
+    });
+  }
+
+  void compute(LGpu &l, int32_t task, micco_stats &st) {
+    const TaskRec &tk = c.tasks[task];
+    const TensorRec &A = c.tensors[tk.a];
+    double2 *pa = l.ptr[tk.a];
+    if (!pa) fail(MICCO_ERR_STATE, "executor: operand not resident");
+    if (tk.kind == TASK_GEMM) {
+      const TensorRec &B = c.tensors[tk.b];
+      double2 *pb = l.ptr[tk.b];
+      if (!pb) fail(MICCO_ERR_STATE, "executor: operand not resident");
+      GemmLayout L;
+      if (!gemm_layout(A.rank, A.dim, B.rank, B.dim, tk.c, tk.pa, tk.pb, L))
+        fail(MICCO_ERR_UNSUPPORTED, "executor: GEMM layout");
+      double2 *pc = alloc(l, bytes_of(tk.out));
+      l.ptr[tk.out] = pc;
+      GemmDesc d{};
+      d.A = pa; d.B = pb; d.C = pc;
+      d.sAt = L.sliceA; d.sBt = L.sliceB; d.sCt = L.sliceC;
+      d.Mo = L.Mo; d.Mi = L.Mi; d.No = L.No; d.Ni = L.Ni; d.Ko = L.Ko; d.Ki = L.Ki;
+      d.sAmo = L.sAmo; d.sAmi = L.sAmi; d.sAko = L.sAko; d.sAki = L.sAki;
+      d.sBko = L.sBko; d.sBki = L.sBki; d.sBno = L.sBno; d.sBni = L.sBni;
+      d.sCmo = L.sCmo; d.sCmi = L.sCmi; d.sCno = L.sCno; d.sCni = L.sCni;
+      d.Lt = c.Lt;
+      d.tilesM = (L.Mi + kGemmBM - 1) / kGemmBM;
+      d.tilesN = (L.Ni + kGemmBN - 1) / kGemmBN;
+      l.gemm.push_back(d);
+      st.gemm_flops += tk.flops;
+    } else {
+      DotLayout L;
+      double2 *pb = nullptr;
+      bool ok;
+      if (tk.kind == TASK_TRACE) {
+        ok = dot_layout(A.rank, A.dim, 0, nullptr, 1, tk.pa, tk.pb, L);
+      } else {
+        const TensorRec &B = c.tensors[tk.b];
+        pb = l.ptr[tk.b];
+        if (!pb) fail(MICCO_ERR_STATE, "executor: operand not resident");
+        ok = dot_layout(A.rank, A.dim, B.rank, B.dim, tk.c, tk.pa, tk.pb, L);
+      }
+      if (!ok) fail(MICCO_ERR_UNSUPPORTED, "executor: dot layout");
+      DotDesc d{};
+      d.A = pa; d.B = pb;
+      d.out = devs[l.dev].scalars + (size_t)c.tensors[tk.out].scalar_slot * c.Lt;
+      d.sAt = L.sliceA; d.sBt = L.sliceB;
+      d.mode = L.mode; d.nO = L.nO; d.X = L.X; d.Y = L.Y;
+      d.sAx = L.sAx; d.sAy = L.sAy; d.sBx = L.sBx; d.sBy = L.sBy;
+      for (int i = 0; i < 3; ++i) { d.O[i] = L.O[i]; d.sAo[i] = L.sAo[i]; d.sBo[i] = L.sBo[i]; }
+      d.Lt = c.Lt;
+      l.dot.push_back(d);
+      st.dot_bytes += (double)(L.sliceA + L.sliceB) * 16.0 * c.Lt;
+    }
+  }
+
+  void run_op(const PlanOp &op, micco_stats &st) {
+    switch (op.kind) {
+      case PlanOp::H2D: {
+        LGpu &l = g[op.gpu];
+        if (!l.local) return;
+        CK(cudaSetDevice(l.dev));
+        auto it = spill_ev.find(op.id);  // a spilled intermediate: wait for its D2H
+        if (it != spill_ev.end() && c.tensors[op.id].node < 0) CK(cudaStreamWaitEvent(l.st, it->second.second, 0));
+        double2 *p = alloc(l, bytes_of(op.id));
+        CK(cudaMemcpyAsync(p, host_src(op.id), bytes_of(op.id), cudaMemcpyHostToDevice, l.st));
+        l.ptr[op.id] = p;
+        st.bytes_h2d += bytes_of(op.id);
+        return;
+      }
+      case PlanOp::P2P: {
+        LGpu &dst = g[op.gpu];
+        LGpu &src = g[op.src];
+        const int64_t nb = bytes_of(op.id);
+        if (dist()) {
+          if (dst.local) {
+            CK(cudaSetDevice(dst.dev));
+            double2 *p = alloc(dst, nb);
+            NK(nccl().Recv(p, (size_t)nb / 8, ncclDouble, op.src, comm, dst.st));
+            dst.ptr[op.id] = p;
+            st.bytes_p2p += nb;
+          } else if (src.local) {
+            CK(cudaSetDevice(src.dev));
+            NK(nccl().Send(src.ptr[op.id], (size_t)nb / 8, ncclDouble, op.gpu, comm, src.st));
+          }
+          return;
+        }
+        cudaEvent_t ready = record(op.src);  // the replica on src is complete
+        CK(cudaSetDevice(dst.dev));
+        CK(cudaStreamWaitEvent(dst.st, ready, 0));
+        double2 *p = alloc(dst, nb);
+        if (dst.dev == src.dev)
+          CK(cudaMemcpyAsync(p, src.ptr[op.id], nb, cudaMemcpyDeviceToDevice, dst.st));
+        else
+          CK(cudaMemcpyPeerAsync(p, dst.dev, src.ptr[op.id], src.dev, nb, dst.st));
+        dst.ptr[op.id] = p;
+        src.readers[op.id].push_back(record(op.gpu));
+        st.bytes_p2p += nb;
+        return;
+      }
+      case PlanOp::SPILL: {
+        LGpu &l = g[op.gpu];
+        if (!l.local) return;
+        CK(cudaSetDevice(l.dev));
+        double *h = spill_arena.alloc(bytes_of(op.id));
+        CK(cudaMemcpyAsync(h, l.ptr[op.id], bytes_of(op.id), cudaMemcpyDeviceToHost, l.st));
+        spill_host[op.id] = h;
+        spill_ev[op.id] = {l.dev, record(op.gpu)};
+        st.bytes_d2h += bytes_of(op.id);
+        return;
+      }
+      case PlanOp::FREE: {
+        if (op.gpu < 0) { spill_host.erase(op.id); spill_ev.erase(op.id); return; }
+        LGpu &l = g[op.gpu];
+        if (!l.local) return;
+        CK(cudaSetDevice(l.dev));
+        auto it = l.readers.find(op.id);
+        if (it != l.readers.end()) {
+          for (cudaEvent_t e : it->second) CK(cudaStreamWaitEvent(l.st, e, 0));
+          l.readers.erase(it);
+        }
+        if (l.ptr[op.id]) CK(cudaFreeAsync(l.ptr[op.id], l.st));
+        l.ptr[op.id] = nullptr;
+        return;
+      }
+      case PlanOp::COMPUTE: {
+        LGpu &l = g[op.gpu];
+        if (!l.local) return;
+        CK(cudaSetDevice(l.dev));
+        compute(l, op.id, st);
+        return;
+      }
+      case PlanOp::FLUSH: {
+        LGpu &l = g[op.gpu];
+        if (!l.local) return;
+        flush(l);
+        return;
+      }
+    }
+  }
+
+  // ---------------------------------------------------------------- execute
+
+  void execute(int n_gpus, const int32_t *bd) {
+    auto t0 = std::chrono::steady_clock::now();
+    setup(n_gpus);
+    for (auto &l : g)
+      if (l.local && l.ptr.size() < c.tensors.size()) l.ptr.resize(c.tensors.size(), nullptr);
+    launches = 0;
+    timed.clear();
+    for (auto &d : devs) { d.sync_events.reset(); d.timing_events.reset(); }
+
+    PlanInput in;
+    in.n_gpus = n;
+    in.policy = c.opt.policy;
+    in.budget = budgets();
+    in.window_graphs = c.opt.window_graphs;
+    in.keep_inputs = c.opt.keep_inputs_resident != 0;
+    in.peer_gbs = (ndev > 1 && !dist()) || dist() ? 700 : 2500;
+    in.host_gbs = 55;
+    in.flops_per_s = 30e12;
+    in.initial_nodes.assign(n, {});
+    for (int i = 0; i < n; ++i) {
+      if (!g[i].local) continue;
+      for (size_t x = 0; x < g[i].ptr.size(); ++x)
+        if (g[i].ptr[x]) in.initial_nodes[i].push_back((int32_t)x);
+    }
+    if (dist() && in.keep_inputs) fail(MICCO_ERR_UNSUPPORTED, "keep_inputs_resident in multi-process mode");
+    Plan plan;
+    if (bd) {
+      for (int i = 0; i < 3; ++i) in.reuse_bound[i] = bd[i];
+      plan = make_plan(c, in);
+    } else if (chosen_bd_n == n) {  // bounds chosen by an earlier sweep for this GPU count
+      for (int i = 0; i < 3; ++i) in.reuse_bound[i] = chosen_bd[i];
+      plan = make_plan(c, in);
+    } else {
+      plan = make_plan_auto(c, in);
+      for (int i = 0; i < 3; ++i) chosen_bd[i] = plan.reuse_bound[i];
+      chosen_bd_n = n;
+    }
+    auto t1 = std::chrono::steady_clock::now();
+
+    micco_stats st{};
+    st.struct_size = sizeof(st);
+    // scalar tables (one per device in use), zeroed before any dot writes
+    const size_t selems = (size_t)std::max(1, c.n_scalar_slots) * c.Lt;
+    std::vector<int> first_lgpu(ndev, -1);
+    for (int i = 0; i < n; ++i)
+      if (g[i].local && first_lgpu[g[i].dev] < 0) first_lgpu[g[i].dev] = i;
+    for (int d = 0; d < ndev; ++d) {
+      if (first_lgpu[d] < 0) continue;
+      LGpu &l = g[first_lgpu[d]];
+      CK(cudaSetDevice(d));
+      if (devs[d].scalar_elems < selems) {
+        CK(cudaStreamSynchronize(l.st));
+        if (devs[d].scalars) CK(cudaFree(devs[d].scalars));
+        CK(cudaMalloc((void **)&devs[d].scalars, selems * sizeof(double2)));
+        devs[d].scalar_elems = selems;
+      }
+      CK(cudaMemsetAsync(devs[d].scalars, 0, selems * sizeof(double2), l.st));
+      cudaEvent_t e = record(first_lgpu[d]);
+      for (int i = 0; i < n; ++i)
+        if (g[i].local && g[i].dev == d && i != first_lgpu[d]) {
+          CK(cudaSetDevice(d));
+          CK(cudaStreamWaitEvent(g[i].st, e, 0));
+        }
+    }
+    for (const PlanOp &op : plan.ops) run_op(op, st);
+    for (auto &l : g)
+      if (l.local && (!l.gemm.empty() || !l.dot.empty())) flush(l);
+    // intermediates must all be released by now; drop leftovers defensively
+    for (auto &l : g) {
+      if (!l.local) continue;
+      CK(cudaSetDevice(l.dev));
+      for (size_t x = 0; x < l.ptr.size(); ++x)
+        if (l.ptr[x] && !(in.keep_inputs && c.tensors[x].node >= 0)) {
+          auto it = l.readers.find((int32_t)x);
+          if (it != l.readers.end())
+            for (cudaEvent_t e : it->second) CK(cudaStreamWaitEvent(l.st, e, 0));
+          CK(cudaFreeAsync(l.ptr[x], l.st));
+          l.ptr[x] = nullptr;
+        }
+      l.readers.clear();
+    }
+
+    // combine devices, finalize on the "home" GPU
+    const int home = dist() ? my_rank() : 0;
+    LGpu &H = g[home];
+    CK(cudaSetDevice(H.dev));
+    for (int i = 0; i < n; ++i)
+      if (i != home && g[i].local) CK(cudaStreamWaitEvent(H.st, record(i), 0));
+    double2 *S = devs[H.dev].scalars;
+    if (dist()) {
+      NK(nccl().AllReduce(S, S, selems * 2, ncclDouble, ncclSum, comm, H.st));
+    } else {
+      for (int d = 0; d < ndev; ++d) {
+        if (d == H.dev || first_lgpu[d] < 0) continue;
+        double2 *tmp = alloc(H, (int64_t)(selems * sizeof(double2)));
+        CK(cudaMemcpyPeerAsync(tmp, H.dev, devs[d].scalars, d, selems * sizeof(double2), H.st));
+        CK(launch_accumulate(S, tmp, (long long)selems, H.st));
+        CK(cudaFreeAsync(tmp, H.st));
+      }
+    }
+    const int G = (int)c.graphs.size();
+    std::vector<int> comp_off(G + 1), comp_slot;
+    std::vector<double2> coefs(G);
+    for (int gi = 0; gi < G; ++gi) {
+      const GraphRec &gr = c.graphs[gi];
+      comp_off[gi] = (int)comp_slot.size();
+      for (int k = gr.comp_begin; k < gr.comp_end; ++k) comp_slot.push_back(c.tensors[c.graph_scalars[k]].scalar_slot);
+      coefs[gi] = make_double2(gr.coef_re, gr.coef_im);
+    }
+    comp_off[G] = (int)comp_slot.size();
+    if (comp_slot.empty()) comp_slot.push_back(0);
+    int *d_off = (int *)alloc(H, (int64_t)comp_off.size() * 4);
+    int *d_slot = (int *)alloc(H, (int64_t)comp_slot.size() * 4);
+    double2 *d_coef = alloc(H, (int64_t)G * 16);
+    CK(cudaMemcpyAsync(d_off, comp_off.data(), comp_off.size() * 4, cudaMemcpyHostToDevice, H.st));
+    CK(cudaMemcpyAsync(d_slot, comp_slot.data(), comp_slot.size() * 4, cudaMemcpyHostToDevice, H.st));
+    CK(cudaMemcpyAsync(d_coef, coefs.data(), (size_t)G * 16, cudaMemcpyHostToDevice, H.st));
+    if (vals_elems < (size_t)G * c.Lt) {
+      CK(cudaStreamSynchronize(H.st));
+      if (d_vals) CK(cudaFree(d_vals));
+      CK(cudaMalloc((void **)&d_vals, (size_t)G * c.Lt * sizeof(double2)));
+      vals_elems = (size_t)G * c.Lt;
+    }
+    if (!h_corr) CK(cudaHostAlloc((void **)&h_corr, 1 << 20, cudaHostAllocPortable));
+    double2 *d_corr = alloc(H, (int64_t)c.Lt * 16);
+    CK(launch_finalize(G, c.Lt, d_off, d_slot, S, d_vals, H.st));
+    CK(launch_correlator_sum(G, c.Lt, d_coef, d_vals, d_corr, H.st));
+    launches += 2;
+    if ((size_t)c.Lt * 16 > (1 << 20)) fail(MICCO_ERR_ARG, "Lt too large");
+    CK(cudaMemcpyAsync(h_corr, d_corr, (size_t)c.Lt * 16, cudaMemcpyDeviceToHost, H.st));
+    CK(cudaFreeAsync(d_off, H.st));
+    CK(cudaFreeAsync(d_slot, H.st));
+    CK(cudaFreeAsync(d_coef, H.st));
+    CK(cudaFreeAsync(d_corr, H.st));
+    for (auto &l : g)
+      if (l.local) { CK(cudaSetDevice(l.dev)); CK(cudaStreamSynchronize(l.st)); }
+    auto t2 = std::chrono::steady_clock::now();
+
+    c.corr.assign(2 * (size_t)c.Lt, 0.0);
+    std::memcpy(c.corr.data(), h_corr, (size_t)c.Lt * 16);
+    spill_host.clear();
+    spill_ev.clear();
+    spill_arena.release_all();
+
+    // statistics
+    for (const Timed &tm : timed) {
+      float ms = 0;
+      CK(cudaSetDevice(tm.dev));
+      CK(cudaEventElapsedTime(&ms, tm.a, tm.b));
+      st.kernel_ms += ms;
+      if (tm.kind == 0) { st.gemm_kernel_ms += ms; ++st.gemm_launches; }
+      else if (tm.kind == 1) { st.dot_kernel_ms += ms; ++st.dot_launches; }
+    }
+    st.wall_ms = std::chrono::duration<double, std::milli>(t2 - t0).count();
+    st.sched_ms = std::chrono::duration<double, std::milli>(t1 - t0).count();
+    st.evictions = plan.evictions;
+    st.cache_hits = plan.cache_hits;
+    st.unique_tasks = (int64_t)c.tasks.size();
+    st.dedup_hits = c.dedup_hits;
+    for (const TaskRec &t : c.tasks) (t.kind == TASK_GEMM ? st.n_gemm : st.n_dot)++;
+    st.n_stages = plan.n_stages;
+    st.kernel_launches = launches;
+    st.flops = plan.flops;
+    for (const GraphRec &gr : c.graphs) st.flops_no_dedup += gr.flops_no_dedup;
+    st.max_over_mean_load = plan.max_over_mean_load;
+    for (int i = 0; i < 3; ++i) st.reuse_bound[i] = plan.reuse_bound[i];
+    st.n_gpus = n;
+    if (dist()) {  // plan-level byte counts are global; report them
+      st.bytes_h2d = plan.bytes_h2d;
+      st.bytes_p2p = plan.bytes_p2p;
+      st.bytes_d2h = plan.bytes_d2h;
+    }
+    c.stats = st;
+  }
+
+  void fetch_graph_values() {
+    const int G = (int)c.graphs.size();
+    c.graph_vals.assign((size_t)G * c.Lt * 2, 0.0);
+    const int home = dist() ? my_rank() : 0;
+    CK(cudaSetDevice(g[home].dev));
+    CK(cudaMemcpy(c.graph_vals.data(), d_vals, (size_t)G * c.Lt * 16, cudaMemcpyDeviceToHost));
+    c.graph_vals_valid = true;
+  }
+
+  void release_cache() {
+    for (auto &l : g) free_lgpu(l, false);
+  }
+};
+
+Executor::Executor(Context &c) : p_(new Impl(c)) {}
+Executor::~Executor() = default;
+void Executor::execute(int n_gpus, const int32_t *bd) { p_->execute(n_gpus, bd); }
+void Executor::fetch_graph_values() { p_->fetch_graph_values(); }
+void Executor::release_cache() { p_->release_cache(); }
+
+}  // namespace micco

@@ -1,0 +1,348 @@
+// kernels.cu — the contraction kernels of the hot path, hand-written for sm_100a.
+//
+// FP64 on B200 has no tcgen05/UMMA kind (ptxas rejects .kind::f64; SURVEY.md §0 probe 2):
+// the FP64 tensor instruction is the warp-level DMMA.8x8x4 (mma.sync m8n8k4 f64), which
+// shares one issue pipe with DFMA.  Measured ceiling on the box: 36.97 TFLOP/s
+// (profiles/fp64_peak_r01.txt).  The GEMM below keeps that pipe fed from a 4-stage
+// cp.async shared-memory pipeline, with 32×32-complex warp tiles (64 independent DMMAs per
+// k-quad per warp, 128 FP64 accumulator registers per thread).
+//
+// Complex arithmetic on the real DMMA: per 8×8×4 complex block,
+//   Cr += Ar·Br + (−Ai)·Bi,   Ci += Ar·Bi + Ai·Br          (4 DMMAs, 8 real flops / complex MAC)
+// with −Ai formed by flipping the sign bit (integer ALU, not the FP64 pipe).  No conjugation
+// anywhere (SURVEY.md §8(c) reading #7).
+#include <cstdio>
+
+#include "kernels.h"
+
+namespace micco {
+namespace {
+
+constexpr int BM = kGemmBM, BN = kGemmBN, BK = kGemmBK, ST = kGemmStages, NT = kGemmThreads;
+constexpr int APITCH = BK + 4;  // complex per A row: 192 B → fragment loads conflict-free
+constexpr int BPITCH = BN + 2;  // complex per B row: 1056 B ≡ 32 (mod 128) → conflict-free
+constexpr int A_STAGE = BM * APITCH;
+constexpr int B_STAGE = BK * BPITCH;
+constexpr int GEMM_SMEM = ST * (A_STAGE + B_STAGE) * 16;
+
+__device__ __forceinline__ void cp_async16(void *smem, const void *gmem, bool valid) {
+  unsigned s = (unsigned)__cvta_generic_to_shared(smem);
+  int sz = valid ? 16 : 0;  // src-size 0 → zero fill (ragged tiles)
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;\n" ::"r"(s), "l"(gmem), "r"(sz));
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() {
+  asm volatile("cp.async.wait_group %0;\n" ::"n"(N));
+}
+
+// D(8x8) += A(8x4, row) · B(4x8, col), FP64 tensor core.
+// Fragments: a = A[lane/4][lane%4], b = B[lane%4][lane/4], d = D[lane/4][2*(lane%4) + {0,1}].
+__device__ __forceinline__ void dmma(double &d0, double &d1, double a, double b) {
+  asm("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};\n"
+      : "+d"(d0), "+d"(d1)
+      : "d"(a), "d"(b));
+}
+
+__device__ __forceinline__ double dneg(double x) {
+  return __longlong_as_double(__double_as_longlong(x) ^ (long long)0x8000000000000000ULL);
+}
+
+template <typename D>
+__device__ __forceinline__ int find_desc(const D *descs, int n, long long item) {
+  int lo = 0, hi = n - 1;
+  while (lo < hi) {
+    int mid = (lo + hi + 1) >> 1;
+    if (descs[mid].tile_begin <= item) lo = mid; else hi = mid - 1;
+  }
+  return lo;
+}
+
+__global__ void __launch_bounds__(NT, 2)
+    zgemm_dmma_kernel(const GemmDesc *__restrict__ descs, int n_desc, long long total) {
+  extern __shared__ __align__(128) double2 smem[];
+  double2 *As = smem;
+  double2 *Bs = smem + ST * A_STAGE;
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int wm = warp >> 1, wn = warp & 1;
+
+  for (long long tile = blockIdx.x; tile < total; tile += gridDim.x) {
+    const GemmDesc &d = descs[find_desc(descs, n_desc, tile)];
+    long long lt = tile - d.tile_begin;
+    const int tn = (int)(lt % d.tilesN); lt /= d.tilesN;
+    const int tm = (int)(lt % d.tilesM); lt /= d.tilesM;
+    const int no = (int)(lt % d.No); lt /= d.No;
+    const int mo = (int)(lt % d.Mo);
+    const int t = (int)(lt / d.Mo);
+    const int m0 = tm * BM, n0 = tn * BN;
+    const int Mi = d.Mi, Ni = d.Ni, Ki = d.Ki;
+    const long long sAmi = d.sAmi, sAki = d.sAki, sBki = d.sBki, sBni = d.sBni;
+    const long long sAko = d.sAko, sBko = d.sBko;
+    const double2 *Abase = d.A + t * d.sAt + mo * d.sAmo + m0 * sAmi;
+    const double2 *Bbase = d.B + t * d.sBt + no * d.sBno + n0 * sBni;
+    const bool a_kfast = (sAki == 1);   // A row-major over (m, k): copy along k
+    const bool b_nfast = (sBni == 1);   // B row-major over (k, n): copy along n
+    const int KT = (Ki + BK - 1) / BK;
+    const int KTOT = d.Ko * KT;
+
+    auto load_stage = [&](int slot, int kt) {
+      const int ko = kt / KT;
+      const int kb = (kt - ko * KT) * BK;
+      const double2 *Ak = Abase + ko * sAko;
+      const double2 *Bk = Bbase + ko * sBko;
+      double2 *as = As + slot * A_STAGE;
+      double2 *bs = Bs + slot * B_STAGE;
+#pragma unroll
+      for (int j = 0; j < (BM * BK) / NT; ++j) {
+        const int e = tid + j * NT;
+        int m, k;
+        if (a_kfast) { k = e & (BK - 1); m = e / BK; } else { m = e & (BM - 1); k = e / BM; }
+        const bool v = (m0 + m < Mi) && (kb + k < Ki);
+        const double2 *src = v ? Ak + (long long)m * sAmi + (long long)(kb + k) * sAki : d.A;
+        cp_async16(as + m * APITCH + k, src, v);
+      }
+#pragma unroll
+      for (int j = 0; j < (BN * BK) / NT; ++j) {
+        const int e = tid + j * NT;
+        int n, k;
+        if (b_nfast) { n = e & (BN - 1); k = e / BN; } else { k = e & (BK - 1); n = e / BK; }
+        const bool v = (n0 + n < Ni) && (kb + k < Ki);
+        const double2 *src = v ? Bk + (long long)(kb + k) * sBki + (long long)n * sBni : d.B;
+        cp_async16(bs + k * BPITCH + n, src, v);
+      }
+    };
+
+    double cr[4][4][2], ci[4][4][2];
+#pragma unroll
+    for (int i = 0; i < 4; ++i)
+#pragma unroll
+      for (int j = 0; j < 4; ++j) { cr[i][j][0] = cr[i][j][1] = ci[i][j][0] = ci[i][j][1] = 0.0; }
+
+#pragma unroll
+    for (int s = 0; s < ST - 1; ++s) {
+      if (s < KTOT) load_stage(s, s);
+      cp_async_commit();
+    }
+    for (int kt = 0; kt < KTOT; ++kt) {
+      cp_async_wait<ST - 2>();
+      __syncthreads();
+      const int nk = kt + ST - 1;
+      if (nk < KTOT) load_stage(nk % ST, nk);
+      cp_async_commit();
+      const double2 *as = As + (kt % ST) * A_STAGE;
+      const double2 *bs = Bs + (kt % ST) * B_STAGE;
+#pragma unroll
+      for (int kq = 0; kq < BK / 4; ++kq) {
+        double ar[4], ai[4], an[4], br[4], bi[4];
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+          const double2 a = as[(wm * 32 + i * 8 + (lane >> 2)) * APITCH + kq * 4 + (lane & 3)];
+          ar[i] = a.x; ai[i] = a.y; an[i] = dneg(a.y);
+        }
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+          const double2 b = bs[(kq * 4 + (lane & 3)) * BPITCH + wn * 32 + j * 8 + (lane >> 2)];
+          br[j] = b.x; bi[j] = b.y;
+        }
+#pragma unroll
+        for (int i = 0; i < 4; ++i)
+#pragma unroll
+          for (int j = 0; j < 4; ++j) {
+            dmma(cr[i][j][0], cr[i][j][1], ar[i], br[j]);
+            dmma(ci[i][j][0], ci[i][j][1], ar[i], bi[j]);
+            dmma(cr[i][j][0], cr[i][j][1], an[i], bi[j]);
+            dmma(ci[i][j][0], ci[i][j][1], ai[i], br[j]);
+          }
+      }
+    }
+    cp_async_wait<0>();
+    __syncthreads();  // the smem ring is reused by the next tile
+
+    double2 *Cbase = d.C + t * d.sCt + mo * d.sCmo + no * d.sCno;
+    const long long sCmi = d.sCmi, sCni = d.sCni;
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      const int m = m0 + wm * 32 + i * 8 + (lane >> 2);
+      if (m >= Mi) continue;
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        const int n = n0 + wn * 32 + j * 8 + (lane & 3) * 2;
+        double2 *cp = Cbase + (long long)m * sCmi + (long long)n * sCni;
+        if (n < Ni) cp[0] = make_double2(cr[i][j][0], ci[i][j][0]);
+        if (n + 1 < Ni) cp[sCni] = make_double2(cr[i][j][1], ci[i][j][1]);
+      }
+    }
+  }
+}
+
+// ---------------------------------------------------------------- dot / trace
+
+constexpr int DT = 256;
+
+__device__ __forceinline__ void cmac(double &sr, double &si, double2 a, double2 b) {
+  sr += a.x * b.x - a.y * b.y;
+  si += a.x * b.y + a.y * b.x;
+}
+
+__global__ void __launch_bounds__(DT) zdot_kernel(const DotDesc *__restrict__ descs, int n_desc) {
+  __shared__ double2 As[32][33], Bs[32][33];
+  __shared__ double red[2][DT / 32];
+  const long long cta = blockIdx.x;
+  int lo = 0, hi = n_desc - 1;
+  while (lo < hi) {
+    int mid = (lo + hi + 1) >> 1;
+    if (descs[mid].cta_begin <= cta) lo = mid; else hi = mid - 1;
+  }
+  const DotDesc &d = descs[lo];
+  const int t = (int)(cta - d.cta_begin);
+  const int tid = threadIdx.x;
+  const double2 *A = d.A + t * d.sAt;
+  const double2 *B = d.B ? d.B + t * d.sBt : nullptr;
+  double sr = 0.0, si = 0.0;
+  const long long O0 = d.O[0], O1 = d.O[1], O2 = d.O[2];
+  const long long Ototal = O0 * O1 * O2;
+  if (d.mode == 2) {
+    for (int i = tid; i < d.X; i += DT) {
+      const double2 a = A[(long long)i * d.sAx];
+      sr += a.x;
+      si += a.y;
+    }
+  } else if (d.mode == 0) {
+    const long long X = d.X, total = Ototal * X;
+    for (long long e = tid; e < total; e += DT) {
+      const long long o = e / X, x = e - o * X;
+      const long long o2 = o % O2, o01 = o / O2, o1 = o01 % O1, o0 = o01 / O1;
+      const long long offA = o0 * d.sAo[0] + o1 * d.sAo[1] + o2 * d.sAo[2] + x * d.sAx;
+      const long long offB = o0 * d.sBo[0] + o1 * d.sBo[1] + o2 * d.sBo[2] + x * d.sBx;
+      cmac(sr, si, A[offA], B[offB]);
+    }
+  } else {  // transpose tiles: A contiguous along x, B contiguous along y
+    const int ty = tid >> 5, tx = tid & 31;
+    for (long long o = 0; o < Ototal; ++o) {
+      const long long o2 = o % O2, o01 = o / O2, o1 = o01 % O1, o0 = o01 / O1;
+      const double2 *Ao = A + o0 * d.sAo[0] + o1 * d.sAo[1] + o2 * d.sAo[2];
+      const double2 *Bo = B + o0 * d.sBo[0] + o1 * d.sBo[1] + o2 * d.sBo[2];
+      for (int y0 = 0; y0 < d.Y; y0 += 32)
+        for (int x0 = 0; x0 < d.X; x0 += 32) {
+          for (int r = ty; r < 32; r += DT / 32) {
+            const int y = y0 + r, x = x0 + tx;
+            As[r][tx] = (y < d.Y && x < d.X) ? Ao[(long long)y * d.sAy + (long long)x * d.sAx] : make_double2(0, 0);
+            const int xb = x0 + r, yb = y0 + tx;
+            Bs[r][tx] = (xb < d.X && yb < d.Y) ? Bo[(long long)xb * d.sBx + (long long)yb * d.sBy] : make_double2(0, 0);
+          }
+          __syncthreads();
+          for (int r = ty; r < 32; r += DT / 32) cmac(sr, si, As[r][tx], Bs[tx][r]);
+          __syncthreads();
+        }
+    }
+  }
+  // deterministic block reduction: xor butterfly, then warps in order
+#pragma unroll
+  for (int off = 16; off > 0; off >>= 1) {
+    sr += __shfl_xor_sync(0xffffffffu, sr, off);
+    si += __shfl_xor_sync(0xffffffffu, si, off);
+  }
+  if ((tid & 31) == 0) { red[0][tid >> 5] = sr; red[1][tid >> 5] = si; }
+  __syncthreads();
+  if (tid == 0) {
+    double ar = 0.0, ai = 0.0;
+    for (int w = 0; w < DT / 32; ++w) { ar += red[0][w]; ai += red[1][w]; }
+    d.out[t] = make_double2(ar, ai);
+  }
+}
+
+// ---------------------------------------------------------------- finalize / sum
+
+__global__ void finalize_kernel(int G, int Lt, const int *__restrict__ comp_off,
+                                const int *__restrict__ comp_slot, const double2 *__restrict__ S,
+                                double2 *__restrict__ vals) {
+  const long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x;
+  if (i >= (long long)G * Lt) return;
+  const int g = (int)(i / Lt), t = (int)(i % Lt);
+  double vr = 1.0, vi = 0.0;
+  for (int c = comp_off[g]; c < comp_off[g + 1]; ++c) {
+    const double2 s = S[(long long)comp_slot[c] * Lt + t];
+    const double nr = vr * s.x - vi * s.y, ni = vr * s.y + vi * s.x;
+    vr = nr;
+    vi = ni;
+  }
+  vals[i] = make_double2(vr, vi);
+}
+
+__global__ void __launch_bounds__(DT) corr_sum_kernel(int G, int Lt, const double2 *__restrict__ coefs,
+                                                      const double2 *__restrict__ vals,
+                                                      double2 *__restrict__ corr) {
+  __shared__ double red[2][DT / 32];
+  const int t = blockIdx.x, tid = threadIdx.x;
+  double sr = 0.0, si = 0.0;
+  for (int g = tid; g < G; g += DT) {
+    const double2 c = coefs[g], v = vals[(long long)g * Lt + t];
+    sr += c.x * v.x - c.y * v.y;
+    si += c.x * v.y + c.y * v.x;
+  }
+#pragma unroll
+  for (int off = 16; off > 0; off >>= 1) {
+    sr += __shfl_xor_sync(0xffffffffu, sr, off);
+    si += __shfl_xor_sync(0xffffffffu, si, off);
+  }
+  if ((tid & 31) == 0) { red[0][tid >> 5] = sr; red[1][tid >> 5] = si; }
+  __syncthreads();
+  if (tid == 0) {
+    double ar = 0.0, ai = 0.0;
+    for (int w = 0; w < DT / 32; ++w) { ar += red[0][w]; ai += red[1][w]; }
+    corr[t] = make_double2(ar, ai);
+  }
+}
+
+__global__ void accumulate_kernel(double2 *dst, const double2 *src, long long n) {
+  for (long long i = blockIdx.x * (long long)blockDim.x + threadIdx.x; i < n;
+       i += (long long)gridDim.x * blockDim.x) {
+    const double2 a = dst[i], b = src[i];
+    dst[i] = make_double2(a.x + b.x, a.y + b.y);
+  }
+}
+
+}  // namespace
+
+cudaError_t launch_gemm_group(const GemmDesc *d_descs, int n, long long total_tiles, cudaStream_t st) {
+  static bool attr_set = false;  // per process; the attribute is per-function, all devices
+  if (!attr_set) {
+    cudaError_t e = cudaFuncSetAttribute(zgemm_dmma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, GEMM_SMEM);
+    if (e != cudaSuccess) return e;
+    attr_set = true;
+  }
+  if (total_tiles <= 0) return cudaSuccess;
+  long long grid = total_tiles < (1LL << 30) ? total_tiles : (1LL << 30);
+  zgemm_dmma_kernel<<<(unsigned)grid, NT, GEMM_SMEM, st>>>(d_descs, n, total_tiles);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_dot_group(const DotDesc *d_descs, int n, long long total_ctas, cudaStream_t st) {
+  if (total_ctas <= 0) return cudaSuccess;
+  zdot_kernel<<<(unsigned)total_ctas, DT, 0, st>>>(d_descs, n);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_finalize(int G, int Lt, const int *comp_off, const int *comp_slot, const double2 *scalars,
+                            double2 *vals, cudaStream_t st) {
+  long long n = (long long)G * Lt;
+  if (n == 0) return cudaSuccess;
+  finalize_kernel<<<(unsigned)((n + 255) / 256), 256, 0, st>>>(G, Lt, comp_off, comp_slot, scalars, vals);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_correlator_sum(int G, int Lt, const double2 *coefs, const double2 *vals, double2 *corr,
+                                  cudaStream_t st) {
+  corr_sum_kernel<<<Lt, DT, 0, st>>>(G, Lt, coefs, vals, corr);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_accumulate(double2 *dst, const double2 *src, long long n, cudaStream_t st) {
+  if (n == 0) return cudaSuccess;
+  long long blocks = (n + 255) / 256;
+  if (blocks > 148 * 16) blocks = 148 * 16;
+  accumulate_kernel<<<(unsigned)blocks, 256, 0, st>>>(dst, src, n);
+  return cudaGetLastError();
+}
+
+}  // namespace micco

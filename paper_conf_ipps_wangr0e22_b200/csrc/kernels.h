@@ -1,0 +1,65 @@
+// kernels.h — device-side task descriptors and launchers of the contraction kernels
+// (sm_100a).  Complex doubles are stored interleaved (double2 = re, im) everywhere on the
+// device, the layout of the C-ABI, so no conversion pass exists.
+#pragma once
+
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace micco {
+
+// A pairwise hadron contraction with a rank >= 1 result, as a batched GEMM over the time
+// slices ("batched matrix multiplications for a meson system or batched
+// tensor contractions for a baryon system"):
+//   C[t][mo,mi][no,ni] = Σ_{ko,ki} A[t][mo,mi][ko,ki] · B[t][ko,ki][no,ni]
+// Every index is split into an outer part (grid / loop) and an inner part (tiled), each
+// with its own stride per tensor, so permuted operand legs (op(A) ∈ {N, T}, baryon legs in
+// any position) are read in place without transposes.  Strides are in complex elements.
+struct GemmDesc {
+  const double2 *A;
+  const double2 *B;
+  double2 *C;
+  long long sAt, sBt, sCt;
+  int Mo, Mi, No, Ni, Ko, Ki;
+  long long sAmo, sAmi, sAko, sAki;
+  long long sBko, sBki, sBno, sBni;
+  long long sCmo, sCmi, sCno, sCni;
+  int Lt, tilesM, tilesN, pad;
+  long long tile_begin;  // first CTA tile of this task in the grouped launch
+};
+
+// The final reduction of two nodes to a scalar per slice ("until
+// only two hadrons are left"), s_t = Σ_idx A[t][idx] · B[t][π(idx)], or a meson trace
+// s_t = Σ_i A[t][i][i] when B == nullptr.
+//   mode 0: x is contiguous in both A and B (flat run of X elements per outer index)
+//   mode 1: x contiguous in A, y contiguous in B → 32×32 shared-memory transpose tiles
+//   mode 2: trace (stride sAx along x)
+struct DotDesc {
+  const double2 *A;
+  const double2 *B;
+  double2 *out;          // out[t], t = 0..Lt-1 (a row of the scalar table)
+  long long sAt, sBt;
+  int mode, nO, X, Y;
+  long long sAx, sAy, sBx, sBy;
+  int O[3], pad0;
+  long long sAo[3], sBo[3];
+  int Lt, pad1;
+  long long cta_begin;   // first CTA of this task in the grouped launch (one CTA per slice)
+};
+
+constexpr int kGemmBM = 64, kGemmBN = 64, kGemmBK = 8, kGemmStages = 4, kGemmThreads = 128;
+
+// Grouped launches: descs in device memory; grid covers total tiles / CTAs.
+cudaError_t launch_gemm_group(const GemmDesc *d_descs, int n, long long total_tiles, cudaStream_t st);
+cudaError_t launch_dot_group(const DotDesc *d_descs, int n, long long total_ctas, cudaStream_t st);
+
+// vals[g][t] = Π_{c in comps(g)} S[slot_c][t] (component scalars)
+cudaError_t launch_finalize(int G, int Lt, const int *comp_off, const int *comp_slot,
+                            const double2 *scalars, double2 *vals, cudaStream_t st);
+// corr[t] = Σ_g coef_g · vals[g][t], fixed-order (deterministic for any GPU count)
+cudaError_t launch_correlator_sum(int G, int Lt, const double2 *coefs, const double2 *vals,
+                                  double2 *corr, cudaStream_t st);
+// dst[i] += src[i] (exact: each slot is nonzero on exactly one source)
+cudaError_t launch_accumulate(double2 *dst, const double2 *src, long long n, cudaStream_t st);
+
+}  // namespace micco

@@ -1,0 +1,331 @@
+// planner.cpp — turns the task DAG into per-GPU operation streams.
+//
+//  * Stages (Fig. 1 L48): graphs are taken in windows (a stream of vectors,
+//    Fig. 6); inside a window a task's stage is its DAG level, so the pairs of one
+//    stage are independent and stages run in order.
+//  * Each pair of a stage is assigned a GPU by the scheduler (Alg. 1/2, scheduler.cpp).
+//  * A per-GPU HBM cache is simulated exactly: an operand is a hit, a peer copy over
+//    NVLink (P2P) or a host upload (H2D); when a GPU would exceed its budget
+//    (GPUMaxMemory, L193) replicas are evicted — dead ones first, then those with another
+//    copy, furthest next use first (the DAG is known, so next use is exact), then sole
+//    copies are spilled to pinned host memory (SURVEY.md §8(c) reading #19; the paper is
+//    silent on the victim, L199/L250).
+//  * Refcounts free intermediates after their last consumer.
+// The output is a flat, globally ordered op list that the executor replays; in
+// multi-process mode every rank builds the identical plan.
+#include <algorithm>
+#include <cmath>
+#include <limits>
+#include <string>
+
+#include "core.h"
+#include "scheduler.h"
+
+namespace micco {
+
+namespace {
+
+struct PlanState {
+  const Context &ctx;
+  const PlanInput &in;
+  Plan &plan;
+  int n;
+  int32_t Lt;
+  std::vector<uint64_t> mask;          // GPUs holding a replica
+  std::vector<char> on_host;           // spilled copy on host (nodes are always on host)
+  std::vector<int32_t> uses_left;
+  std::vector<std::vector<int32_t>> use_stages;  // sorted stage ids where the tensor is an operand
+  std::vector<std::vector<int32_t>> res;         // resident tensors per GPU
+  std::vector<std::vector<int32_t>> res_pos;     // index in res[g], -1 if absent
+  std::vector<std::vector<int32_t>> pin;         // pin epoch per GPU per tensor
+  std::vector<int32_t> epoch;
+  std::vector<int64_t> mem;
+  std::vector<double> st_flops, st_h2d, st_p2p, st_d2h;
+  int32_t stage = 0;
+
+  PlanState(const Context &c, const PlanInput &i, Plan &p)
+      : ctx(c), in(i), plan(p), n(i.n_gpus), Lt(c.Lt) {}
+
+  int64_t bytes(int32_t x) const { return ctx.tensors[x].bytes(Lt); }
+  bool is_node(int32_t x) const { return ctx.tensors[x].node >= 0; }
+
+  void add_res(int g, int32_t x) {
+    res_pos[g][x] = (int32_t)res[g].size();
+    res[g].push_back(x);
+    mask[x] |= 1ULL << g;
+    mem[g] += bytes(x);
+    plan.gpu_peak_bytes[g] = std::max(plan.gpu_peak_bytes[g], mem[g]);
+  }
+  void drop_res(int g, int32_t x) {
+    int32_t i = res_pos[g][x];
+    int32_t last = res[g].back();
+    res[g][i] = last;
+    res_pos[g][last] = i;
+    res[g].pop_back();
+    res_pos[g][x] = -1;
+    mask[x] &= ~(1ULL << g);
+    mem[g] -= bytes(x);
+  }
+  void emit(PlanOp::Kind k, int g, int src, int32_t id) { plan.ops.push_back(PlanOp{k, g, src, id}); }
+
+  int32_t next_use(int32_t x) const {
+    const auto &u = use_stages[x];
+    auto it = std::lower_bound(u.begin(), u.end(), stage);
+    return it == u.end() ? std::numeric_limits<int32_t>::max() : *it;
+  }
+
+  // Evict unpinned replicas on g until need more bytes fit; false if impossible.
+  bool make_room(int g, int64_t need) {
+    const int64_t budget = in.budget[g];
+    if (mem[g] + need <= budget) return true;
+    struct Cand { int cls; int32_t next; int32_t x; };
+    std::vector<Cand> cands;
+    for (int32_t x : res[g]) {
+      if (pin[g][x] == epoch[g]) continue;
+      int cls;
+      if (uses_left[x] == 0) cls = 0;
+      else if (is_node(x) || on_host[x] || (mask[x] & ~(1ULL << g))) cls = 1;
+      else cls = 2;
+      cands.push_back({cls, next_use(x), x});
+    }
+    std::sort(cands.begin(), cands.end(), [](const Cand &a, const Cand &b) {
+      if (a.cls != b.cls) return a.cls < b.cls;
+      if (a.next != b.next) return a.next > b.next;
+      return a.x < b.x;
+    });
+    for (const Cand &c : cands) {
+      if (mem[g] + need <= budget) break;
+      if (c.cls == 2) {  // sole copy: spill to pinned host memory first
+        emit(PlanOp::SPILL, g, -1, c.x);
+        on_host[c.x] = 1;
+        plan.bytes_d2h += bytes(c.x);
+        st_d2h[g] += (double)bytes(c.x);
+      }
+      emit(PlanOp::FREE, g, -1, c.x);
+      drop_res(g, c.x);
+      ++plan.evictions;
+    }
+    return mem[g] + need <= budget;
+  }
+
+  void fetch(int g, int32_t x) {
+    uint64_t others = mask[x] & ~(1ULL << g);
+    if (others) {  // a peer holds it: NVLink peer copy
+      int src = __builtin_ctzll(others);
+      emit(PlanOp::P2P, g, src, x);
+      plan.bytes_p2p += bytes(x);
+      st_p2p[g] += (double)bytes(x);
+    } else {
+      if (!is_node(x) && !on_host[x]) fail(MICCO_ERR_STATE, "planner: lost the only copy of a tensor");
+      emit(PlanOp::H2D, g, -1, x);
+      plan.bytes_h2d += bytes(x);
+      st_h2d[g] += (double)bytes(x);
+    }
+    add_res(g, x);
+  }
+
+  void release(int32_t x) {  // last consumer done
+    if (is_node(x) && in.keep_inputs) return;  // stays cached (dead → evicted first)
+    for (uint64_t m = mask[x]; m; m &= m - 1) {
+      int g = __builtin_ctzll(m);
+      emit(PlanOp::FREE, g, -1, x);
+      drop_res(g, x);
+    }
+    if (!is_node(x) && on_host[x]) {
+      emit(PlanOp::FREE, -1, -1, x);  // release the host spill copy
+      on_host[x] = 0;
+    }
+  }
+};
+
+}  // namespace
+
+Plan make_plan(const Context &ctx, const PlanInput &in) {
+  Plan plan;
+  const int n = in.n_gpus;
+  plan.n_gpus = n;
+  for (int i = 0; i < 3; ++i) plan.reuse_bound[i] = in.reuse_bound[i];
+  const int32_t T = (int32_t)ctx.tasks.size(), NT = (int32_t)ctx.tensors.size();
+  const int32_t G = (int32_t)ctx.graphs.size();
+  plan.task_gpu.assign(T, -1);
+  plan.gpu_peak_bytes.assign(n, 0);
+  plan.gpu_flops.assign(n, 0.0);
+
+  // 1. window of every task = window of the first graph that needs it
+  const int32_t W = in.window_graphs > 0 ? in.window_graphs : 256;
+  std::vector<int32_t> task_window(T, -1);
+  std::vector<int32_t> stack;
+  for (int32_t g = 0; g < G; ++g) {
+    const int32_t w = g / W;
+    for (int32_t c = ctx.graphs[g].comp_begin; c < ctx.graphs[g].comp_end; ++c) {
+      int32_t t0 = ctx.tensors[ctx.graph_scalars[c]].task;
+      if (t0 >= 0 && task_window[t0] < 0) { task_window[t0] = w; stack.push_back(t0); }
+      while (!stack.empty()) {
+        int32_t t = stack.back();
+        stack.pop_back();
+        for (int32_t op : {ctx.tasks[t].a, ctx.tasks[t].b}) {
+          if (op < 0) continue;
+          int32_t pt = ctx.tensors[op].task;
+          if (pt >= 0 && task_window[pt] < 0) { task_window[pt] = w; stack.push_back(pt); }
+        }
+      }
+    }
+  }
+  // 2. stages = (window, level), tasks in id order inside a stage
+  std::vector<int32_t> order;
+  order.reserve(T);
+  for (int32_t t = 0; t < T; ++t)
+    if (task_window[t] >= 0) order.push_back(t);
+  std::stable_sort(order.begin(), order.end(), [&](int32_t x, int32_t y) {
+    if (task_window[x] != task_window[y]) return task_window[x] < task_window[y];
+    return ctx.tasks[x].level < ctx.tasks[y].level;
+  });
+  std::vector<std::pair<int32_t, int32_t>> stages;  // [begin, end) in order
+  for (size_t i = 0; i < order.size();) {
+    size_t j = i;
+    while (j < order.size() && task_window[order[j]] == task_window[order[i]] &&
+           ctx.tasks[order[j]].level == ctx.tasks[order[i]].level)
+      ++j;
+    stages.push_back({(int32_t)i, (int32_t)j});
+    i = j;
+  }
+
+  PlanState S(ctx, in, plan);
+  S.mask.assign(NT, 0);
+  S.on_host.assign(NT, 0);
+  S.uses_left.assign(NT, 0);
+  S.use_stages.assign(NT, {});
+  for (int32_t s = 0; s < (int32_t)stages.size(); ++s)
+    for (int32_t i = stages[s].first; i < stages[s].second; ++i) {
+      const TaskRec &tk = ctx.tasks[order[i]];
+      for (int32_t op : {tk.a, tk.b}) {
+        if (op < 0 || (op == tk.b && tk.b == tk.a)) continue;
+        ++S.uses_left[op];
+        if (S.use_stages[op].empty() || S.use_stages[op].back() != s) S.use_stages[op].push_back(s);
+      }
+    }
+  S.res.assign(n, {});
+  S.res_pos.assign(n, std::vector<int32_t>(NT, -1));
+  S.pin.assign(n, std::vector<int32_t>(NT, -1));
+  S.epoch.assign(n, 0);
+  S.mem.assign(n, 0);
+  S.st_flops.assign(n, 0);
+  S.st_h2d.assign(n, 0);
+  S.st_p2p.assign(n, 0);
+  S.st_d2h.assign(n, 0);
+  for (int g = 0; g < n && g < (int)in.initial_nodes.size(); ++g)
+    for (int32_t x : in.initial_nodes[g])
+      if (x >= 0 && x < NT && !((S.mask[x] >> g) & 1)) S.add_res(g, x);
+
+  Scheduler sched(n, in.policy, in.reuse_bound, in.budget);
+  std::vector<std::vector<int32_t>> chunk(n);
+  auto flush = [&](int g) {
+    for (int32_t t : chunk[g]) S.emit(PlanOp::COMPUTE, g, -1, t);
+    S.emit(PlanOp::FLUSH, g, -1, -1);
+    chunk[g].clear();
+    ++S.epoch[g];
+  };
+
+  double predicted = 0;
+  for (int32_t s = 0; s < (int32_t)stages.size(); ++s) {
+    S.stage = s;
+    sched.begin_vector(stages[s].second - stages[s].first);
+    std::fill(S.st_flops.begin(), S.st_flops.end(), 0.0);
+    std::fill(S.st_h2d.begin(), S.st_h2d.end(), 0.0);
+    std::fill(S.st_p2p.begin(), S.st_p2p.end(), 0.0);
+    std::fill(S.st_d2h.begin(), S.st_d2h.end(), 0.0);
+    for (int32_t i = stages[s].first; i < stages[s].second; ++i) {
+      const int32_t t = order[i];
+      const TaskRec &tk = ctx.tasks[t];
+      const int32_t a = tk.a, b = tk.b;
+      const bool same = (b < 0 || b == a);
+      const TensorRec &out = ctx.tensors[tk.out];
+      SchedPair p;
+      p.m1 = S.mask[a];
+      p.m2 = same ? S.mask[a] : S.mask[b];
+      p.same = same;
+      p.b1 = S.bytes(a);
+      p.b2 = same ? 0 : S.bytes(b);
+      p.bout = out.rank > 0 ? S.bytes(tk.out) : 0;
+      p.flops = tk.flops;
+      sched.mem = S.mem;
+      const int g = sched.decide(p);
+      const uint64_t bit = 1ULL << g;
+      auto need_bytes = [&]() {
+        int64_t need = p.bout;
+        if (!(S.mask[a] & bit)) need += p.b1;
+        if (!same && !(S.mask[b] & bit)) need += p.b2;
+        return need;
+      };
+      // pin operands so the eviction below never drops them
+      S.pin[g][a] = S.epoch[g];
+      if (!same) S.pin[g][b] = S.epoch[g];
+      if (!S.make_room(g, need_bytes())) {
+        flush(g);  // split the stage: run what is pinned, then retry with this pair only
+        S.pin[g][a] = S.epoch[g];
+        if (!same) S.pin[g][b] = S.epoch[g];
+        if (!S.make_room(g, need_bytes()))
+          fail(MICCO_ERR_OOM, "planner: one contraction's operands and output (" +
+                                  std::to_string(need_bytes()) + " B) exceed the GPU budget (" +
+                                  std::to_string(in.budget[g]) + " B)");
+      }
+      if (S.mask[a] & bit) ++plan.cache_hits; else S.fetch(g, a);
+      if (!same) { if (S.mask[b] & bit) ++plan.cache_hits; else S.fetch(g, b); }
+      if (out.rank > 0) {
+        S.add_res(g, tk.out);
+        S.pin[g][tk.out] = S.epoch[g];
+      }
+      sched.account(g, p);
+      plan.task_gpu[t] = g;
+      plan.gpu_flops[g] += tk.flops;
+      plan.flops += tk.flops;
+      S.st_flops[g] += tk.flops;
+      chunk[g].push_back(t);
+    }
+    for (int g = 0; g < n; ++g)
+      if (!chunk[g].empty()) flush(g);
+    // release operands whose last consumer ran
+    for (int32_t i = stages[s].first; i < stages[s].second; ++i) {
+      const TaskRec &tk = ctx.tasks[order[i]];
+      for (int32_t op : {tk.a, tk.b}) {
+        if (op < 0 || (op == tk.b && tk.b == tk.a)) continue;
+        if (--S.uses_left[op] == 0) S.release(op);
+      }
+    }
+    double worst = 0;
+    for (int g = 0; g < n; ++g) {
+      double tg = S.st_flops[g] / in.flops_per_s + (S.st_h2d[g] + S.st_d2h[g]) / (in.host_gbs * 1e9) +
+                  S.st_p2p[g] / (in.peer_gbs * 1e9);
+      worst = std::max(worst, tg);
+    }
+    predicted += worst;
+  }
+  plan.n_stages = (int64_t)stages.size();
+  plan.predicted_s = predicted;
+  double mx = 0, sum = 0;
+  for (double f : plan.gpu_flops) { mx = std::max(mx, f); sum += f; }
+  plan.max_over_mean_load = sum > 0 ? mx / (sum / n) : 1.0;
+  return plan;
+}
+
+Plan make_plan_auto(const Context &ctx, PlanInput in) {
+  if (in.n_gpus == 1 || in.policy == MICCO_POLICY_ROUND_ROBIN || in.policy == MICCO_POLICY_LEAST_LOADED ||
+      in.policy == MICCO_POLICY_MICCO_NAIVE) {
+    for (int i = 0; i < 3; ++i) in.reuse_bound[i] = 0;
+    return make_plan(ctx, in);
+  }
+  // Sweep {0,1,2}^3 (a superset of the paper's 13 sets, L355) through
+  // the planner's cost model and keep the cheapest plan (ties: lexicographically smallest).
+  Plan best;
+  bool have = false;
+  for (int b0 = 0; b0 < 3; ++b0)
+    for (int b1 = 0; b1 < 3; ++b1)
+      for (int b2 = 0; b2 < 3; ++b2) {
+        in.reuse_bound[0] = b0; in.reuse_bound[1] = b1; in.reuse_bound[2] = b2;
+        Plan p = make_plan(ctx, in);
+        if (!have || p.predicted_s < best.predicted_s * (1 - 1e-12)) { best = std::move(p); have = true; }
+      }
+  return best;
+}
+
+}  // namespace micco

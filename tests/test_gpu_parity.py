@@ -1,0 +1,163 @@
+"""GPU parity: the CUDA path (through the C-ABI) against the CPU oracle on the
+same seeded inputs (task rule ③).  Tolerance: ≤ 1e-10 relative per time slice
+(BASELINE.json north_star); bit-exact for exact-integer inputs (SURVEY.md §8(c)
+"Bit-exact GPU parity"); bitwise-identical C(t) across GPU counts, policies,
+reuse bounds, windows and budgets (§8(e))."""
+import numpy as np
+import pytest
+
+import oracle
+import paper_conf_ipps_wangr0e22_b200 as M
+from micco_inputs import workloads
+from micco_inputs.gen import GraphSpec, MODE_INT3, NodeSpec, Workload
+
+pytestmark = pytest.mark.gpu
+
+TOL = 1e-10
+
+
+def run_gpu(wl, n_gpus=1, reuse_bound=None, **kw):
+    ctx = M.Context(**kw)
+    M.load_workload(ctx, wl)
+    ctx.execute(n_gpus, reuse_bound)
+    C = ctx.correlator()
+    vals = np.array([[ctx.graph_value(g, t) for t in range(wl.Lt)] for g in range(len(wl.graphs))])
+    st = ctx.stats()
+    ctx.close()
+    return C, vals, st
+
+
+def rel_err(a, b):
+    return np.max(np.abs(a - b) / np.maximum(np.abs(b), 1e-300))
+
+
+def check(wl, **kw):
+    C, vals, st = run_gpu(wl, **kw)
+    Co, valso = oracle.correlator(wl, return_values=True)
+    assert rel_err(C, Co) <= TOL, (rel_err(C, Co), st)
+    for g in range(len(wl.graphs)):
+        assert rel_err(vals[g], valso[g]) <= TOL, g
+    return C, st
+
+
+def test_c1_parity():
+    C, st = check(workloads.c1_two_meson())
+    assert st["kernel_launches"] > 0 and st["n_gemm"] > 0
+
+
+def test_c1_integer_bit_exact():
+    wl = workloads.c1_two_meson(mode=MODE_INT3)
+    C, vals, _ = run_gpu(wl)
+    Co, valso = oracle.correlator(wl, return_values=True)
+    assert np.array_equal(vals, valso)
+    assert np.array_equal(C, Co)
+
+
+@pytest.mark.parametrize("N", [1, 3, 33, 64, 100, 130, 257])
+def test_meson_chains_ragged_shapes(N):
+    """Cycles of 1..5 mesons with random transposes (all N/T operand layouts), at
+    sizes that leave ragged GEMM tiles and K tails."""
+    rng = np.random.default_rng(N)
+    nodes = [NodeSpec(2, N, 900 + i) for i in range(5)]
+    graphs = []
+    for k in (1, 2, 3, 4, 5):
+        for _ in range(2):
+            inst = [int(x) for x in rng.integers(0, 5, size=k)]
+            flips = [bool(x) for x in rng.integers(0, 2, size=k)]
+            graphs.append(GraphSpec(inst, workloads.meson_cycle_edges(k, flips),
+                                    [int(x) for x in rng.permutation(k)], complex(rng.choice([-1.0, 1.0]))))
+    wl = Workload(f"ragged{N}", 3, 77, 0, nodes, graphs)
+    check(wl)
+    wl_int = Workload(f"ragged{N}i", 3, 77, MODE_INT3, nodes, graphs)
+    C, vals, _ = run_gpu(wl_int)
+    Co, valso = oracle.correlator(wl_int, return_values=True)
+    assert np.array_equal(vals, valso)
+
+
+@pytest.mark.parametrize("N", [2, 3, 5])
+def test_tiny_random_graphs_with_baryons(N):
+    wl = workloads.tiny_random(seed=100 + N, n_graphs=40, N=N, Lt=3)
+    check(wl)
+    check(wl, window_graphs=7)
+
+
+@pytest.mark.parametrize("order", ["greedy", "chain"])
+def test_two_baryon_all_matchings(order):
+    """All 720 leg matchings of a two-baryon correlator (rank-3 GETT, c = 1 and
+    c = 2, rank-3 dots with every permutation), N = 9 (ragged), Lt = 2."""
+    wl = workloads.c4_two_baryon(n_combos=1, N=9, Lt=2, pool=2, order=order)
+    check(wl)
+    wli = workloads.c4_two_baryon(n_combos=1, N=9, Lt=2, pool=2, order=order, mode=MODE_INT3)
+    C, vals, _ = run_gpu(wli)
+    Co, valso = oracle.correlator(wli, return_values=True)
+    assert np.array_equal(vals, valso)
+
+
+def test_two_baryon_n64_sample():
+    """C4 at its full tensor size (N = 64 baryons), a sample of matchings, Lt = 4."""
+    wl = workloads.c4_two_baryon(n_combos=1, N=64, Lt=4, pool=2, order="chain",
+                                 matchings=list(range(0, 720, 97)))
+    check(wl)
+
+
+def test_cross_run_invariance_bitwise():
+    """C(t) is bitwise identical for any GPU count, policy, reuse bound, window and
+    budget (the scalar table is exact-summed; finalize is fixed-order)."""
+    wl = workloads.c2_meson_set(n_graphs=120, N=24, Lt=4, rate=0.6, dist="gaussian", flips=True)
+    ref, _, _ = run_gpu(wl, 1)
+    Co = oracle.correlator(wl)
+    assert rel_err(ref, Co) <= TOL
+    node_bytes = 24 * 24 * 4 * 16
+    for n in (2, 3, 4, 8):
+        for pol in ("micco", "round_robin", "least_loaded", "micco_naive"):
+            C, _, _ = run_gpu(wl, n, [1, 2, 0] if pol == "micco" else None, policy=pol, window_graphs=16)
+            assert np.array_equal(C, ref), (n, pol)
+    for bd in ([0, 0, 0], [2, 2, 2], None):
+        C, _, _ = run_gpu(wl, 4, bd)
+        assert np.array_equal(C, ref)
+    # memory pressure: evictions and host spills
+    C, _, st = run_gpu(wl, 2, [1, 1, 1], mem_budget_bytes=10 * node_bytes, window_graphs=40)
+    assert st["evictions"] > 0
+    assert np.array_equal(C, ref)
+
+
+def test_keep_inputs_resident_repeat():
+    wl = workloads.c2_meson_set(n_graphs=60, N=32, Lt=4, rate=0.8)
+    ctx = M.Context(keep_inputs_resident=True)
+    M.load_workload(ctx, wl)
+    ctx.execute(1)
+    C1 = ctx.correlator()
+    s1 = ctx.stats()
+    ctx.execute(1)
+    C2 = ctx.correlator()
+    s2 = ctx.stats()
+    assert np.array_equal(C1, C2)
+    assert s1["bytes_h2d"] > 0 and s2["bytes_h2d"] == 0
+    ctx.release_cache()
+    ctx.execute(1)
+    assert np.array_equal(ctx.correlator(), C1)
+    ctx.close()
+
+
+def test_c2_bench_config_sampled():
+    """C2 at its full sizes (N = 128, Lt = 64) in the bench's launch configuration
+    (windows of 256 graphs, grouped launches), 1000 graphs; sampled graph values
+    against the oracle computed one by one."""
+    wl = workloads.c2_meson_set(n_graphs=1000, N=128, Lt=64, rate=0.9)
+    ctx = M.Context()
+    M.load_workload(ctx, wl)
+    ctx.execute(1)
+    rng = np.random.default_rng(0)
+    sample = sorted(int(x) for x in rng.choice(len(wl.graphs), 6, replace=False))
+    sub = wl.subset(sample)
+    _, valso = oracle.correlator(sub, return_values=True)
+    for i, g in enumerate(sample):
+        v = np.array([ctx.graph_value(g, t) for t in range(wl.Lt)])
+        assert rel_err(v, valso[i]) <= TOL, g
+    ctx.close()
+
+
+def test_c3_sampled_n256():
+    """C3 meson wirings at N = 256 (the multi-meson config's tensor size), Lt = 4."""
+    wl = workloads.c3_multi_meson(n_graphs=40, N=256, Lt=4, pool=4)
+    check(wl.subset(list(range(12))))

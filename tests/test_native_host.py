@@ -1,0 +1,205 @@
+"""Host-side tests of libmicco.so that need no GPU: the library loads and exports
+every symbol include/micco.h declares; the builder's validation, dedup and
+hash-consing; the planner's invariants; and the native scheduler against the
+oracle (oracle/sched.py) decision for decision."""
+import re
+from pathlib import Path
+
+import numpy as np
+import pytest
+
+import paper_conf_ipps_wangr0e22_b200 as M
+from micco_inputs import workloads
+from micco_inputs.gen import GraphSpec, NodeSpec, Workload
+from oracle.sched import MiccoSchedulerOracle, Pair
+
+ROOT = Path(__file__).resolve().parent.parent
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _built():
+    import sys
+    sys.path.insert(0, str(ROOT / "tools"))
+    from build import build_lib
+    build_lib()
+
+
+def test_exports_every_declared_symbol():
+    hdr = (ROOT / "include" / "micco.h").read_text()
+    declared = set(re.findall(r"MICCO_API\s+[\w\s\*]+?\b(micco_\w+)\s*\(", hdr))
+    assert declared == set(M.EXPORTS), declared ^ set(M.EXPORTS)
+    L = M.lib()
+    for name in declared:
+        assert hasattr(L, name), name
+
+
+def _ctx(**kw):
+    kw.setdefault("mem_budget_bytes", 1 << 30)
+    return M.Context(**kw)
+
+
+def test_node_dedup_by_content_and_lt_check():
+    ctx = _ctx()
+    a = np.arange(2 * 4 * 4, dtype=np.float64).reshape(2, 4, 4) + 1j
+    i0 = ctx.add_node(a)
+    i1 = ctx.add_node(a.copy())
+    i2 = ctx.add_node(a + 1)
+    assert i0 == i1 and i2 != i0
+    with pytest.raises(M.MiccoError) as e:
+        ctx.add_node(np.zeros((3, 4, 4), dtype=complex))
+    assert e.value.status == -1  # Lt mismatch
+
+
+def test_graph_validation_errors():
+    ctx = _ctx()
+    m = ctx.add_node(np.ones((1, 2, 2), dtype=complex))
+    b = ctx.add_node(np.ones((1, 2, 2, 2), dtype=complex))
+    cases = [
+        ([m, m], [(0, 1, 1, 0)], None, -3),                      # unmatched legs
+        ([m, m], [(0, 1, 1, 0), (0, 1, 1, 1)], None, -3),        # leg matched twice
+        ([m, m], [(0, 2, 1, 0), (1, 1, 0, 0)], None, -3),        # leg index >= rank
+        ([m, m], [(0, 1, 1, 0), (1, 1, 0, 0)], [0, 0], -3),      # order not a permutation
+        ([b], [(0, 0, 0, 1)], None, -3),                          # odd legs
+        ([b, m], [(0, 0, 0, 1), (0, 2, 1, 0), (1, 1, 1, 0)], None, -3),
+    ]
+    for inst, edges, order, code in cases:
+        with pytest.raises(M.MiccoError) as e:
+            ctx.add_graph(inst, edges, order)
+        assert e.value.status == code, (edges, e.value)
+    # baryon partial trace is unsupported
+    with pytest.raises(M.MiccoError) as e:
+        ctx.add_graph([b, m, b], [(0, 0, 0, 1), (0, 2, 1, 0), (1, 1, 2, 0), (2, 1, 2, 2)])
+    assert e.value.status in (-3, -4)
+    # a failing graph leaves no tasks behind
+    st, _ = ctx.plan(1, [0, 0, 0]) if ctx.n_graphs else ({"unique_tasks": 0}, None)
+
+
+def test_unequal_N_rejected():
+    ctx = _ctx()
+    a = ctx.add_node(np.ones((1, 2, 2), dtype=complex))
+    b = ctx.add_node(np.ones((1, 3, 3), dtype=complex))
+    with pytest.raises(M.MiccoError) as e:
+        ctx.add_graph([a, b], [(0, 1, 1, 0), (1, 1, 0, 0)])
+    assert e.value.status == -3
+
+
+def test_hash_consing_counts():
+    """tr(AB), tr(ABC), tr(ABD): the product A·B is one task shared by the last two
+    (overlapping reduction paths), and tr(AB) is a dot."""
+    ctx = _ctx()
+    rng = np.random.default_rng(0)
+    ids = [ctx.add_node(rng.standard_normal((1, 4, 4)) + 0j) for _ in range(4)]
+    A, B, C, D = ids
+    ctx.add_graph([A, B], workloads.meson_cycle_edges(2), [0, 1])
+    ctx.add_graph([A, B, C], workloads.meson_cycle_edges(3), [0, 1, 2])
+    ctx.add_graph([A, B, D], workloads.meson_cycle_edges(3), [0, 1, 2])
+    st, _ = ctx.plan(1, [0, 0, 0])
+    # tasks: dot(A,B), gemm(A,B), dot(AB,C), dot(AB,D)
+    assert st["unique_tasks"] == 4 and st["n_gemm"] == 1 and st["n_dot"] == 3
+    assert st["dedup_hits"] == 1
+    # identical graph again: everything is a hit
+    ctx.add_graph([A, B, C], workloads.meson_cycle_edges(3), [0, 1, 2])
+    st2, _ = ctx.plan(1, [0, 0, 0])
+    assert st2["unique_tasks"] == 4 and st2["dedup_hits"] == 3
+
+
+def test_flops_accounting():
+    """N×N×N complex GEMM = 8N³ flops per slice."""
+    N, Lt = 8, 3
+    ctx = _ctx()
+    rng = np.random.default_rng(1)
+    ids = [ctx.add_node(rng.standard_normal((Lt, N, N)) + 0j) for _ in range(3)]
+    ctx.add_graph(ids, workloads.meson_cycle_edges(3), [0, 1, 2])
+    st, _ = ctx.plan(1, [0, 0, 0])
+    assert st["flops"] == 8 * N ** 3 * Lt + 8 * N * N * Lt
+    assert st["flops_no_dedup"] == st["flops"]
+
+
+def test_plan_stage_structure_and_invariants():
+    wl = workloads.c2_meson_set(n_graphs=300, N=8, Lt=2, rate=0.5)
+    ctx = _ctx(window_graphs=50)
+    M.load_workload(ctx, wl)
+    for n in (1, 2, 4, 8):
+        st, assign = ctx.plan(n, [1, 1, 1], n_tasks=None)
+        assert st["n_gpus"] == n
+        st, assign = M.micco_plan(ctx.h, n, [1, 1, 1], n_tasks=st["unique_tasks"])
+        assert np.all((assign >= 0) & (assign < n))  # every task assigned exactly once
+        if n == 1:
+            assert st["bytes_p2p"] == 0 and st["max_over_mean_load"] == 1.0
+    # 6 windows × up to 3 levels
+    assert st["n_stages"] <= 6 * 3
+
+
+def test_tight_budget_forces_evictions_and_spills():
+    wl = workloads.c2_meson_set(n_graphs=200, N=16, Lt=4, rate=0.7)
+    node_bytes = 16 * 16 * 4 * 16
+    big = _ctx(mem_budget_bytes=1 << 30, window_graphs=200)
+    M.load_workload(big, wl)
+    s_big, _ = big.plan(1, [0, 0, 0])
+    small = _ctx(mem_budget_bytes=12 * node_bytes, window_graphs=200)
+    M.load_workload(small, wl)
+    s_small, _ = small.plan(1, [0, 0, 0])
+    assert s_big["evictions"] == 0
+    assert s_small["evictions"] > 0
+    assert s_small["bytes_h2d"] > s_big["bytes_h2d"]
+    # a budget below one task's working set is an OOM error
+    tiny = _ctx(mem_budget_bytes=2 * node_bytes)
+    M.load_workload(tiny, wl)
+    with pytest.raises(M.MiccoError) as e:
+        tiny.plan(1, [0, 0, 0])
+    assert e.value.status == -5
+
+
+def test_reuse_beats_round_robin_on_repetition_heavy_set():
+    """On a repetition-heavy set MICCO moves fewer bytes than round-robin
+    (BASELINE.json north_star; Fig. 2 L90)."""
+    wl = workloads.c2_meson_set(n_graphs=600, N=16, Lt=4, rate=0.9, dist="gaussian")
+    res = {}
+    for pol in ("micco", "round_robin", "least_loaded", "micco_naive"):
+        ctx = _ctx(policy=pol, window_graphs=64)
+        M.load_workload(ctx, wl)
+        st, _ = ctx.plan(4, [1, 2, 0] if pol == "micco" else None)
+        res[pol] = st["bytes_h2d"] + st["bytes_p2p"]
+    assert res["micco"] < res["round_robin"]
+    assert res["micco"] <= res["micco_naive"]
+
+
+def test_auto_bounds_sweep_picks_a_valid_set():
+    wl = workloads.c2_meson_set(n_graphs=200, N=8, Lt=2, rate=0.8)
+    ctx = _ctx(window_graphs=32)
+    M.load_workload(ctx, wl)
+    st, _ = ctx.plan(4, None)
+    assert all(0 <= b <= 2 for b in st["reuse_bound"])
+
+
+# ---------------------------------------------------------------- scheduler parity with the oracle
+
+
+def _random_stream(rng, n_gpus, n_vec=6, n_tensors=40):
+    vecs, nxt = [], 10_000
+    for _ in range(n_vec):
+        v = []
+        for _ in range(int(rng.integers(1, 30))):
+            t1, t2 = int(rng.integers(0, n_tensors)), int(rng.integers(0, n_tensors))
+            fl = float(rng.integers(1, 5)) * 1e6
+            v.append((t1, t2, nxt, fl, int(rng.integers(1, 4)) * 100, int(rng.integers(1, 4)) * 100, 100))
+            nxt += 1
+        vecs.append(v)
+    res = [(int(rng.integers(0, n_tensors)), int(rng.integers(0, n_gpus))) for _ in range(int(rng.integers(0, 20)))]
+    return vecs, res
+
+
+@pytest.mark.parametrize("seed", range(30))
+def test_native_scheduler_matches_oracle(seed):
+    rng = np.random.default_rng(seed)
+    n = int(rng.integers(1, 9))
+    bd = [int(x) for x in rng.integers(0, 3, size=3)]
+    budget = float(rng.choice([1e30, 3000.0, 8000.0]))
+    vecs, res = _random_stream(rng, n)
+    O = MiccoSchedulerOracle(n, bd, budget)
+    for t, g in res:
+        if g not in O.res.setdefault(t, set()):
+            O.res[t].add(g)
+    got_o = O.run([[Pair(*p) for p in v] for v in vecs])
+    got_n = M.micco_debug_schedule(n, bd, budget, vecs, resident=res)
+    assert got_n == got_o
