@@ -177,6 +177,7 @@ struct Plan {
   int64_t n_stages = 0;
   double flops = 0, max_over_mean_load = 1, predicted_s = 0;
   std::vector<double> gpu_flops;
+  std::vector<std::pair<int32_t, uint64_t>> final_nodes;  // (node tensor, GPU mask) left cached
 };
 
 struct PlanInput {

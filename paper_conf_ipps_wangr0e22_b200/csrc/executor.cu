@@ -164,6 +164,7 @@ struct Executor::Impl {
   std::vector<ncclComm_t> comms_all;  // single-process multi-device
   std::vector<int64_t> budget_cache;
   int budget_cache_n = 0;
+  std::vector<std::pair<int32_t, uint64_t>> cached_nodes;
   int32_t chosen_bd[3] = {0, 0, 0};
   int chosen_bd_n = 0;
   // results on device 0
@@ -219,6 +220,7 @@ struct Executor::Impl {
     if (ndev < 1) fail(MICCO_ERR_CUDA, "no CUDA device (micco has no CPU fallback)");
     if (n_gpus == n && !g.empty()) return;
     teardown();
+    cached_nodes.clear();
     n = n_gpus;
     devs.assign(ndev, DevState{});
     for (int d = 0; d < ndev; ++d) {
@@ -538,13 +540,16 @@ struct Executor::Impl {
     in.peer_gbs = (ndev > 1 && !dist()) || dist() ? 700 : 2500;
     in.host_gbs = 55;
     in.flops_per_s = 30e12;
+    // node replicas cached by the previous execute: the previous plan's final residency,
+    // identical on every rank (the local pointers must agree with it)
     in.initial_nodes.assign(n, {});
-    for (int i = 0; i < n; ++i) {
-      if (!g[i].local) continue;
-      for (size_t x = 0; x < g[i].ptr.size(); ++x)
-        if (g[i].ptr[x]) in.initial_nodes[i].push_back((int32_t)x);
-    }
-    if (dist() && in.keep_inputs) fail(MICCO_ERR_UNSUPPORTED, "keep_inputs_resident in multi-process mode");
+    if (in.keep_inputs)
+      for (const auto &fn : cached_nodes)
+        for (int i = 0; i < n; ++i)
+          if ((fn.second >> i) & 1) {
+            if (g[i].local && !g[i].ptr[fn.first]) fail(MICCO_ERR_STATE, "executor: cache out of sync");
+            in.initial_nodes[i].push_back(fn.first);
+          }
     Plan plan;
     if (bd) {
       for (int i = 0; i < 3; ++i) in.reuse_bound[i] = bd[i];
@@ -557,6 +562,7 @@ struct Executor::Impl {
       for (int i = 0; i < 3; ++i) chosen_bd[i] = plan.reuse_bound[i];
       chosen_bd_n = n;
     }
+    cached_nodes = plan.final_nodes;
     auto t1 = std::chrono::steady_clock::now();
 
     micco_stats st{};
@@ -706,6 +712,7 @@ struct Executor::Impl {
 
   void release_cache() {
     for (auto &l : g) free_lgpu(l, false);
+    cached_nodes.clear();
   }
 };
 

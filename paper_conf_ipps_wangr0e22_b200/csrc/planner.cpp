@@ -300,6 +300,9 @@ Plan make_plan(const Context &ctx, const PlanInput &in) {
     }
     predicted += worst;
   }
+  if (in.keep_inputs)
+    for (int32_t x = 0; x < NT; ++x)
+      if (S.mask[x] && ctx.tensors[x].node >= 0) plan.final_nodes.push_back({x, S.mask[x]});
   plan.n_stages = (int64_t)stages.size();
   plan.predicted_s = predicted;
   double mx = 0, sum = 0;
