@@ -299,9 +299,9 @@ def main():
                      "traffic": traffic, "gemm_launches": gemm_launches,
                      "gemm_share_of_step": gemm_ms / sum(step_ms)},
         "cpu_baseline": cpu,
-        "e2e": {"value": G / (statistics.mean(e2e_ms) / 1e3), "unit": "graphs/s",
-                "h2d_bytes_per_step": int(statistics.mean(e2e_h2d)), "d2h_bytes_per_step": int(e2e_d2h[0]),
-                "ms_per_step": statistics.mean(e2e_ms)},
+        "e2e": ({"value": G / (statistics.mean(e2e_ms) / 1e3), "unit": "graphs/s",
+                 "h2d_bytes_per_step": int(statistics.mean(e2e_h2d)), "d2h_bytes_per_step": int(e2e_d2h[0]),
+                 "ms_per_step": statistics.mean(e2e_ms)} if e2e_ms else None),
         "gpu_launches": launches,
         "clocks": clk,
         "sched_ms_per_step": statistics.mean(s["sched_ms"] for s in stats),
