@@ -395,6 +395,9 @@ struct Executor::Impl {
       GemmLayout L;
       if (!gemm_layout(A.rank, A.dim, B.rank, B.dim, tk.c, tk.pa, tk.pb, L))
         fail(MICCO_ERR_UNSUPPORTED, "executor: GEMM layout");
+      const long long lim = (1LL << 31) - 1;  // the GEMM keeps per-slice offsets in 32 bits
+      if (L.sliceA > lim || L.sliceB > lim || L.sliceC > lim)
+        fail(MICCO_ERR_UNSUPPORTED, "executor: tensor slice exceeds 2^31 elements");
       double2 *pc = alloc(l, bytes_of(tk.out));
       l.ptr[tk.out] = pc;
       GemmDesc d{};

@@ -12,6 +12,7 @@
 // with −Ai formed by flipping the sign bit (integer ALU, not the FP64 pipe).  No conjugation
 // anywhere (SURVEY.md §8(c) reading #7).
 #include <cstdio>
+#include <cstdlib>
 
 #include "kernels.h"
 
@@ -175,6 +176,216 @@ __global__ void __launch_bounds__(NT, 2)
   }
 }
 
+// ---------------------------------------------------------------- persistent GEMM (v2)
+//
+// Same math and warp tiling as zgemm_dmma_kernel, restructured to remove the per-tile
+// bubbles the round-1 ncu capture showed (profiles/ncu_gemm_r01.json: long-scoreboard
+// stalls at tile prologues and descriptor loads):
+//  * persistent: grid = resident CTAs; CTA c owns a contiguous range of tiles, so its task
+//    descriptor changes rarely and is advanced linearly (no per-tile binary search);
+//  * one continuous cp.async pipeline over the CTA's whole (tile, k-step) sequence: the
+//    loads of the next tile are in flight while the current tile finishes and writes back;
+//  * BK = 16 with 3 stages (half the barriers per tile), per-thread 32-bit element offsets
+//    precomputed once per tile.
+constexpr int BK2 = 16, ST2 = 3;
+constexpr int APITCH2 = BK2 + 4;  // 320 B ≡ 64 (mod 128): A fragment loads conflict-free
+constexpr int BPITCH2 = BN + 2;   // 1056 B ≡ 32 (mod 128)
+constexpr int A_STAGE2 = BM * APITCH2;
+constexpr int B_STAGE2 = BK2 * BPITCH2;
+constexpr int GEMM2_SMEM = ST2 * (A_STAGE2 + B_STAGE2) * 16;
+constexpr int LPT = (BM * BK2) / NT;  // elements per thread per operand per stage (8)
+
+struct LoadCur {
+  const double2 *A, *B;  // tile bases (t, mo/no, m0/n0 applied)
+  long long sAko, sBko;
+  int sAki, sBki;
+  int Ki, KT, KTOT;
+  int offA[LPT], offB[LPT];
+  unsigned vA, vB;       // m-valid / n-valid bit per element
+  bool akf, bnf;
+};
+
+struct StoreCur {
+  double2 *C;
+  int sCmi, sCni, Mi, Ni, m0, n0, KTOT;
+};
+
+__device__ __forceinline__ void decode_tile(const GemmDesc *__restrict__ descs, int n_desc, int &task,
+                                            long long tile, int tid, LoadCur *L, StoreCur *S) {
+  while (task + 1 < n_desc && descs[task + 1].tile_begin <= tile) ++task;
+  const GemmDesc &d = descs[task];
+  long long lt = tile - d.tile_begin;
+  const int tilesN = d.tilesN, tilesM = d.tilesM, No = d.No, Mo = d.Mo;
+  const int tn = (int)(lt % tilesN); lt /= tilesN;
+  const int tm = (int)(lt % tilesM); lt /= tilesM;
+  const int no = (int)(lt % No); lt /= No;
+  const int mo = (int)(lt % Mo);
+  const long long t = lt / Mo;
+  const int m0 = tm * BM, n0 = tn * BN;
+  const int KT = (d.Ki + BK2 - 1) / BK2;
+  if (L) {
+    const int sAmi = (int)d.sAmi, sAki = (int)d.sAki, sBki = (int)d.sBki, sBni = (int)d.sBni;
+    L->A = d.A + t * d.sAt + mo * d.sAmo + (long long)m0 * sAmi;
+    L->B = d.B + t * d.sBt + no * d.sBno + (long long)n0 * sBni;
+    L->sAko = d.sAko; L->sBko = d.sBko; L->sAki = sAki; L->sBki = sBki;
+    L->Ki = d.Ki; L->KT = KT; L->KTOT = d.Ko * KT;
+    L->akf = (sAki == 1);
+    L->bnf = (sBni == 1);
+    const int Mi = d.Mi, Ni = d.Ni;
+    L->vA = 0; L->vB = 0;
+#pragma unroll
+    for (int j = 0; j < LPT; ++j) {
+      const int e = tid + j * NT;
+      int m, k, n, kb;
+      if (L->akf) { k = e & (BK2 - 1); m = e / BK2; } else { m = e & (BM - 1); k = e / BM; }
+      L->offA[j] = m * sAmi + k * sAki;
+      if (m0 + m < Mi) L->vA |= 1u << j;
+      if (L->bnf) { n = e & (BN - 1); kb = e / BN; } else { kb = e & (BK2 - 1); n = e / BK2; }
+      L->offB[j] = kb * sBki + n * sBni;
+      if (n0 + n < Ni) L->vB |= 1u << j;
+    }
+  }
+  if (S) {
+    S->C = d.C + t * d.sCt + mo * d.sCmo + no * d.sCno;
+    S->sCmi = (int)d.sCmi; S->sCni = (int)d.sCni;
+    S->Mi = d.Mi; S->Ni = d.Ni; S->m0 = m0; S->n0 = n0;
+    S->KTOT = d.Ko * KT;
+  }
+}
+
+__global__ void __launch_bounds__(NT, 2)
+    zgemm_dmma_persistent(const GemmDesc *__restrict__ descs, int n_desc, long long total) {
+  extern __shared__ __align__(128) double2 smem[];
+  double2 *As = smem;
+  double2 *Bs = smem + ST2 * A_STAGE2;
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int wm = warp >> 1, wn = warp & 1;
+
+  const long long per = total / gridDim.x, rem = total % gridDim.x;
+  const long long t_begin = blockIdx.x * per + min((long long)blockIdx.x, rem);
+  const long long t_end = t_begin + per + ((long long)blockIdx.x < rem ? 1 : 0);
+  if (t_begin >= t_end) return;
+
+  int task_l = 0, task_c = 0;
+  {  // first task by binary search, then linear advance
+    int lo = 0, hi = n_desc - 1;
+    while (lo < hi) {
+      int mid = (lo + hi + 1) >> 1;
+      if (descs[mid].tile_begin <= t_begin) lo = mid; else hi = mid - 1;
+    }
+    task_l = task_c = lo;
+  }
+  LoadCur L;
+  StoreCur S;
+  long long tile_l = t_begin, tile_c = t_begin;
+  int kt_l = 0, kt_c = 0;
+  decode_tile(descs, n_desc, task_l, tile_l, tid, &L, nullptr);
+  decode_tile(descs, n_desc, task_c, tile_c, tid, nullptr, &S);
+  bool more_l = true;
+
+  auto issue_load = [&](int slot) {
+    const int ko = kt_l / L.KT;
+    const int kb = (kt_l - ko * L.KT) * BK2;
+    const double2 *Ak = L.A + ko * L.sAko + (long long)kb * L.sAki;
+    const double2 *Bk = L.B + ko * L.sBko + (long long)kb * L.sBki;
+    double2 *as = As + slot * A_STAGE2;
+    double2 *bs = Bs + slot * B_STAGE2;
+#pragma unroll
+    for (int j = 0; j < LPT; ++j) {
+      const int e = tid + j * NT;
+      int m, k;
+      if (L.akf) { k = e & (BK2 - 1); m = e / BK2; } else { m = e & (BM - 1); k = e / BM; }
+      const bool v = ((L.vA >> j) & 1u) && (kb + k < L.Ki);
+      cp_async16(as + m * APITCH2 + k, v ? Ak + L.offA[j] : L.A, v);
+    }
+#pragma unroll
+    for (int j = 0; j < LPT; ++j) {
+      const int e = tid + j * NT;
+      int n, k;
+      if (L.bnf) { n = e & (BN - 1); k = e / BN; } else { k = e & (BK2 - 1); n = e / BK2; }
+      const bool v = ((L.vB >> j) & 1u) && (kb + k < L.Ki);
+      cp_async16(bs + k * BPITCH2 + n, v ? Bk + L.offB[j] : L.B, v);
+    }
+    // advance the load cursor (possibly into the next tile)
+    if (++kt_l == L.KTOT) {
+      kt_l = 0;
+      if (++tile_l < t_end) decode_tile(descs, n_desc, task_l, tile_l, tid, &L, nullptr);
+      else more_l = false;
+    }
+  };
+
+  double cr[4][4][2], ci[4][4][2];
+#pragma unroll
+  for (int i = 0; i < 4; ++i)
+#pragma unroll
+    for (int j = 0; j < 4; ++j) { cr[i][j][0] = cr[i][j][1] = ci[i][j][0] = ci[i][j][1] = 0.0; }
+
+#pragma unroll
+  for (int s = 0; s < ST2 - 1; ++s) {
+    if (more_l) issue_load(s);
+    cp_async_commit();
+  }
+  int slot_c = 0, slot_l = ST2 - 1;
+  for (;;) {
+    cp_async_wait<ST2 - 2>();
+    __syncthreads();
+    if (more_l) issue_load(slot_l);
+    cp_async_commit();
+    slot_l = (slot_l + 1 == ST2) ? 0 : slot_l + 1;
+    const double2 *as = As + slot_c * A_STAGE2;
+    const double2 *bs = Bs + slot_c * B_STAGE2;
+#pragma unroll
+    for (int kq = 0; kq < BK2 / 4; ++kq) {
+      double ar[4], ai[4], an[4], br[4], bi[4];
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {
+        const double2 a = as[(wm * 32 + i * 8 + (lane >> 2)) * APITCH2 + kq * 4 + (lane & 3)];
+        ar[i] = a.x; ai[i] = a.y; an[i] = dneg(a.y);
+      }
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        const double2 b = bs[(kq * 4 + (lane & 3)) * BPITCH2 + wn * 32 + j * 8 + (lane >> 2)];
+        br[j] = b.x; bi[j] = b.y;
+      }
+#pragma unroll
+      for (int i = 0; i < 4; ++i)
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+          dmma(cr[i][j][0], cr[i][j][1], ar[i], br[j]);
+          dmma(ci[i][j][0], ci[i][j][1], ar[i], bi[j]);
+        }
+#pragma unroll
+      for (int i = 0; i < 4; ++i)
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+          dmma(cr[i][j][0], cr[i][j][1], an[i], bi[j]);
+          dmma(ci[i][j][0], ci[i][j][1], ai[i], br[j]);
+        }
+    }
+    slot_c = (slot_c + 1 == ST2) ? 0 : slot_c + 1;
+    if (++kt_c == S.KTOT) {  // tile done: write back (next tile's loads already in flight)
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {
+        const int m = S.m0 + wm * 32 + i * 8 + (lane >> 2);
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+          const int n = S.n0 + wn * 32 + j * 8 + (lane & 3) * 2;
+          if (m < S.Mi) {
+            double2 *cp = S.C + (long long)m * S.sCmi + (long long)n * S.sCni;
+            if (n < S.Ni) cp[0] = make_double2(cr[i][j][0], ci[i][j][0]);
+            if (n + 1 < S.Ni) cp[S.sCni] = make_double2(cr[i][j][1], ci[i][j][1]);
+          }
+          cr[i][j][0] = cr[i][j][1] = ci[i][j][0] = ci[i][j][1] = 0.0;
+        }
+      }
+      kt_c = 0;
+      if (++tile_c >= t_end) break;
+      decode_tile(descs, n_desc, task_c, tile_c, tid, nullptr, &S);
+    }
+  }
+  cp_async_wait<0>();
+}
+
 // ---------------------------------------------------------------- dot / trace
 
 constexpr int DT = 256;
@@ -306,14 +517,30 @@ __global__ void accumulate_kernel(double2 *dst, const double2 *src, long long n)
 
 cudaError_t launch_gemm_group(const GemmDesc *d_descs, int n, long long total_tiles, cudaStream_t st) {
   static bool attr_set = false;  // per process; the attribute is per-function, all devices
+  static int use_v1 = -1;
+  if (use_v1 < 0) {
+    const char *e = getenv("MICCO_GEMM_V1");
+    use_v1 = (e && e[0] == '1') ? 1 : 0;
+  }
   if (!attr_set) {
     cudaError_t e = cudaFuncSetAttribute(zgemm_dmma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, GEMM_SMEM);
+    if (e != cudaSuccess) return e;
+    e = cudaFuncSetAttribute(zgemm_dmma_persistent, cudaFuncAttributeMaxDynamicSharedMemorySize, GEMM2_SMEM);
     if (e != cudaSuccess) return e;
     attr_set = true;
   }
   if (total_tiles <= 0) return cudaSuccess;
-  long long grid = total_tiles < (1LL << 30) ? total_tiles : (1LL << 30);
-  zgemm_dmma_kernel<<<(unsigned)grid, NT, GEMM_SMEM, st>>>(d_descs, n, total_tiles);
+  if (use_v1) {
+    long long grid = total_tiles < (1LL << 30) ? total_tiles : (1LL << 30);
+    zgemm_dmma_kernel<<<(unsigned)grid, NT, GEMM_SMEM, st>>>(d_descs, n, total_tiles);
+    return cudaGetLastError();
+  }
+  int dev = 0, sms = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  long long grid = 2LL * sms;  // 2 resident CTAs per SM (248 registers, 112 KB smem each)
+  if (grid > total_tiles) grid = total_tiles;
+  zgemm_dmma_persistent<<<(unsigned)grid, NT, GEMM2_SMEM, st>>>(d_descs, n, total_tiles);
   return cudaGetLastError();
 }
 
