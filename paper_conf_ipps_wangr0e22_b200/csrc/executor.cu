@@ -136,7 +136,9 @@ struct Timed {
 struct LGpu {
   int idx = 0, dev = 0;
   bool local = true;
-  cudaStream_t st = nullptr;
+  cudaStream_t st = nullptr;   // compute stream: kernels, P2P, spills, frees
+  cudaStream_t cst = nullptr;  // copy stream: H2D prefetch (async, overlaps the kernels)
+  std::vector<cudaEvent_t> flush_ev;  // compute-stream event after each flushed chunk
   std::vector<double2 *> ptr;                                  // tensor → replica
   std::unordered_map<int32_t, std::vector<cudaEvent_t>> readers;  // peer reads to wait for before free
   std::vector<GemmDesc> gemm;
@@ -204,6 +206,7 @@ struct Executor::Impl {
     for (auto &p : l.ptr)
       if (p) { cudaFreeAsync(p, l.st); p = nullptr; }
     cudaStreamSynchronize(l.st);
+    if (l.cst) cudaStreamSynchronize(l.cst);
     l.readers.clear();
     if (destroy_stream) {
       for (int i = 0; i < kRingSlots; ++i)
@@ -211,7 +214,9 @@ struct Executor::Impl {
       if (l.ring_h) cudaFreeHost(l.ring_h);
       if (l.ring_d) cudaFree(l.ring_d);
       cudaStreamDestroy(l.st);
+      cudaStreamDestroy(l.cst);
       l.st = nullptr;
+      l.cst = nullptr;
     }
   }
 
@@ -255,6 +260,7 @@ struct Executor::Impl {
         devs[l.dev].init = true;
       }
       CK(cudaStreamCreateWithFlags(&l.st, cudaStreamNonBlocking));
+      CK(cudaStreamCreateWithFlags(&l.cst, cudaStreamNonBlocking));
       CK(cudaHostAlloc((void **)&l.ring_h, kRingSlots * kSlotBytes, cudaHostAllocPortable));
       CK(cudaMalloc((void **)&l.ring_d, kRingSlots * kSlotBytes));
       for (int s = 0; s < kRingSlots; ++s) CK(cudaEventCreateWithFlags(&l.ring_ev[s], cudaEventDisableTiming));
@@ -335,7 +341,7 @@ struct Executor::Impl {
   }
 
   template <typename D, typename Launch>
-  void launch_batch(LGpu &l, std::vector<D> &v, int kind, Launch &&launch) {
+  void launch_batch(LGpu &l, std::vector<D> &v, int kind, int cls, Launch &&prefix) {
     if (v.empty()) return;
     const size_t per = kSlotBytes / sizeof(D);
     for (size_t i0 = 0; i0 < v.size(); i0 += per) {
@@ -343,15 +349,14 @@ struct Executor::Impl {
       int slot;
       char *h = ring_slot(l, cnt * sizeof(D), slot);
       std::memcpy(h, &v[i0], cnt * sizeof(D));
-      long long first = 0, total = 0;
       D *hd = (D *)h;
-      launch(hd, (int)cnt, first, total);  // fixes offsets in the staged copy
+      const long long total = prefix(hd, (int)cnt);  // grid offsets in the staged copy
       char *dptr = l.ring_d + (size_t)slot * kSlotBytes;
       CK(cudaMemcpyAsync(dptr, h, cnt * sizeof(D), cudaMemcpyHostToDevice, l.st));
       CK(cudaEventRecord(l.ring_ev[slot], l.st));
       Timed tm{devs[l.dev].timing_events.get(), devs[l.dev].timing_events.get(), kind, l.dev};
       CK(cudaEventRecord(tm.a, l.st));
-      if (kind == 0) CK(launch_gemm_group((const GemmDesc *)dptr, (int)cnt, total, l.st));
+      if (kind == 0) CK(launch_gemm_group((const GemmDesc *)dptr, (int)cnt, total, cls, l.st));
       else CK(launch_dot_group((const DotDesc *)dptr, (int)cnt, total, l.st));
       CK(cudaEventRecord(tm.b, l.st));
       timed.push_back(tm);
@@ -362,24 +367,27 @@ struct Executor::Impl {
 
   void flush(LGpu &l) {
     CK(cudaSetDevice(l.dev));
-    launch_batch(l, l.gemm, 0, [](GemmDesc *d, int cnt, long long &first, long long &total) {
-      long long acc = 0;
-      for (int i = 0; i < cnt; ++i) {
-        long long tiles = (long long)d[i].Lt * d[i].Mo * d[i].No * d[i].tilesM * d[i].tilesN;
-        d[i].tile_begin = acc;
-        acc += tiles;
-      }
-      first = 0;
-      total = acc;
-    });
-    launch_batch(l, l.dot, 1, [](DotDesc *d, int cnt, long long &first, long long &total) {
+    if (!l.gemm.empty()) {  // one grouped launch per operand-layout class
+      std::vector<GemmDesc> by[kGemmClasses];
+      for (const GemmDesc &d : l.gemm) by[d.cls].push_back(d);
+      l.gemm.clear();
+      for (int c = 0; c < kGemmClasses; ++c)
+        launch_batch(l, by[c], 0, c, [](GemmDesc *d, int cnt) {
+          long long acc = 0;
+          for (int i = 0; i < cnt; ++i) {
+            d[i].tile_begin = acc;
+            acc += (long long)d[i].Lt * d[i].Mo * d[i].No * d[i].tilesM * d[i].tilesN;
+          }
+          return acc;
+        });
+    }
+    launch_batch(l, l.dot, 1, 0, [](DotDesc *d, int cnt) {
       long long acc = 0;
       for (int i = 0; i < cnt; ++i) {
         d[i].cta_begin = acc;
         acc += d[i].Lt;
       }
-      first = 0;
-      total = acc;
+      return acc;
     });
   }
 
@@ -410,6 +418,7 @@ struct Executor::Impl {
       d.Lt = c.Lt;
       d.tilesM = (L.Mi + kGemmBM - 1) / kGemmBM;
       d.tilesN = (L.Ni + kGemmBN - 1) / kGemmBN;
+      d.cls = gemm_layout_class(d);
       l.gemm.push_back(d);
       st.gemm_flops += tk.flops;
     } else {
@@ -441,14 +450,24 @@ struct Executor::Impl {
   void run_op(const PlanOp &op, micco_stats &st) {
     switch (op.kind) {
       case PlanOp::H2D: {
+        // Prefetch on the copy stream (NEXT #1 of SURVEY.md §8(f); "asynchronous
+        // data copy and prefetching"): the copy for chunk k+1 may start once chunk k-1 has
+        // finished (bounded look-ahead keeps the pool within the planned budget + one chunk);
+        // the compute stream waits for the copy right away, so everything it enqueues later
+        // (kernels, peer reads) sees the data, while already-enqueued kernels keep running.
         LGpu &l = g[op.gpu];
         if (!l.local) return;
         CK(cudaSetDevice(l.dev));
+        if (l.flush_ev.size() >= 2) CK(cudaStreamWaitEvent(l.cst, l.flush_ev[l.flush_ev.size() - 2], 0));
         auto it = spill_ev.find(op.id);  // a spilled intermediate: wait for its D2H
-        if (it != spill_ev.end() && c.tensors[op.id].node < 0) CK(cudaStreamWaitEvent(l.st, it->second.second, 0));
-        double2 *p = alloc(l, bytes_of(op.id));
-        CK(cudaMemcpyAsync(p, host_src(op.id), bytes_of(op.id), cudaMemcpyHostToDevice, l.st));
-        l.ptr[op.id] = p;
+        if (it != spill_ev.end() && c.tensors[op.id].node < 0) CK(cudaStreamWaitEvent(l.cst, it->second.second, 0));
+        void *p = nullptr;
+        CK(cudaMallocAsync(&p, (size_t)bytes_of(op.id), l.cst));
+        CK(cudaMemcpyAsync(p, host_src(op.id), bytes_of(op.id), cudaMemcpyHostToDevice, l.cst));
+        cudaEvent_t done = devs[l.dev].sync_events.get();
+        CK(cudaEventRecord(done, l.cst));
+        CK(cudaStreamWaitEvent(l.st, done, 0));
+        l.ptr[op.id] = (double2 *)p;
         st.bytes_h2d += bytes_of(op.id);
         return;
       }
@@ -518,6 +537,7 @@ struct Executor::Impl {
         LGpu &l = g[op.gpu];
         if (!l.local) return;
         flush(l);
+        l.flush_ev.push_back(record(op.gpu));
         return;
       }
     }
@@ -532,6 +552,7 @@ struct Executor::Impl {
       if (l.local && l.ptr.size() < c.tensors.size()) l.ptr.resize(c.tensors.size(), nullptr);
     launches = 0;
     timed.clear();
+    for (auto &l : g) l.flush_ev.clear();
     for (auto &d : devs) { d.sync_events.reset(); d.timing_events.reset(); }
 
     PlanInput in;
@@ -664,7 +685,11 @@ struct Executor::Impl {
     CK(cudaFreeAsync(d_coef, H.st));
     CK(cudaFreeAsync(d_corr, H.st));
     for (auto &l : g)
-      if (l.local) { CK(cudaSetDevice(l.dev)); CK(cudaStreamSynchronize(l.st)); }
+      if (l.local) {
+        CK(cudaSetDevice(l.dev));
+        CK(cudaStreamSynchronize(l.st));
+        CK(cudaStreamSynchronize(l.cst));
+      }
     auto t2 = std::chrono::steady_clock::now();
 
     c.corr.assign(2 * (size_t)c.Lt, 0.0);

@@ -386,6 +386,280 @@ __global__ void __launch_bounds__(NT, 2)
   cp_async_wait<0>();
 }
 
+// ---------------------------------------------------------------- warp-specialized GEMM (v3)
+//
+// Producer/consumer split so the DMMA warps execute nothing but shared-memory fragment loads
+// and DMMAs (the v1/v2 captures show long-scoreboard stalls from the cp.async address math
+// and register reuse inside the DMMA warps):
+//  * warp 4 (producer) streams tile rows with 1-D bulk async copies
+//    (cp.async.bulk ... mbarrier::complete_tx, SASS UBLKCP) into padded shared-memory rows,
+//    zero-filling ragged rows/tails itself, and signals a "full" mbarrier per stage;
+//  * warps 0-3 (consumers) wait on "full", run the 32×32-complex DMMA warp tiles, release
+//    the stage on an "empty" mbarrier, and write C from registers at the end of each tile;
+//  * persistent CTAs over contiguous tile ranges; the pipeline runs across tile boundaries.
+// The smem orientation follows the global one (A [m][k] or [k][m], B [k][n] or [n][k]) so
+// every bulk copy is a contiguous run; the fragment loads are specialised per orientation
+// (all four are bank-conflict free with the pitches below).  Operands with no unit-stride
+// inner index use zgemm_dmma_kernel.
+
+constexpr int NCW = 4;                    // consumer warps
+constexpr int NT3 = (NCW + 1) * 32;       // + 1 producer warp
+constexpr int PITCH_MK = BK2 + 4;         // [m][k] / [n][k]: 320 B rows
+constexpr int PITCH_KM = BM + 2;          // [k][m] / [k][n]: 1056 B rows
+
+template <bool A_MK, bool B_KN>
+struct V3Cfg {
+  static constexpr int A_ELEMS = A_MK ? BM * PITCH_MK : BK2 * PITCH_KM;
+  static constexpr int B_ELEMS = B_KN ? BK2 * PITCH_KM : BN * PITCH_MK;
+  static constexpr int STAGE = A_ELEMS + B_ELEMS;
+  static constexpr int ST = (220 * 1024) / (STAGE * 16) > 6 ? 6 : (220 * 1024) / (STAGE * 16);
+  static constexpr int SMEM = ST * STAGE * 16 + 2 * ST * 8;
+};
+
+__device__ __forceinline__ uint32_t smem_u32(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
+
+__device__ __forceinline__ void mbar_init(uint32_t bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;\n" ::"r"(bar), "r"(count));
+}
+__device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
+  uint32_t done;
+  do {
+    asm volatile(
+        "{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n selp.u32 %0, 1, 0, p;\n}\n"
+        : "=r"(done)
+        : "r"(bar), "r"(parity)
+        : "memory");
+  } while (!done);
+}
+__device__ __forceinline__ void mbar_arrive(uint32_t bar) {
+  asm volatile("{\n .reg .b64 st;\n mbarrier.arrive.shared::cta.b64 st, [%0];\n}\n" ::"r"(bar) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_tx(uint32_t bar, uint32_t bytes) {
+  asm volatile("{\n .reg .b64 st;\n mbarrier.arrive.expect_tx.shared::cta.b64 st, [%0], %1;\n}\n" ::"r"(bar),
+               "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void bulk_g2s(uint32_t dst, const void *src, uint32_t bytes, uint32_t bar) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];\n" ::"r"(dst),
+               "l"(src), "r"(bytes), "r"(bar)
+               : "memory");
+}
+
+struct V3Tile {  // what both roles need about one tile
+  const GemmDesc *d;
+  long long t;
+  int mo, no, m0, n0, KT, KTOT;
+};
+
+__device__ __forceinline__ void v3_decode(const GemmDesc *__restrict__ descs, int n_desc, int &task, long long tile,
+                                          V3Tile &T) {
+  while (task + 1 < n_desc && descs[task + 1].tile_begin <= tile) ++task;
+  const GemmDesc *d = descs + task;
+  long long lt = tile - d->tile_begin;
+  const int tilesN = d->tilesN, tilesM = d->tilesM, No = d->No, Mo = d->Mo;
+  const int tn = (int)(lt % tilesN); lt /= tilesN;
+  const int tm = (int)(lt % tilesM); lt /= tilesM;
+  T.no = (int)(lt % No); lt /= No;
+  T.mo = (int)(lt % Mo);
+  T.t = lt / Mo;
+  T.m0 = tm * BM;
+  T.n0 = tn * BN;
+  T.d = d;
+  T.KT = (d->Ki + BK2 - 1) / BK2;
+  T.KTOT = d->Ko * T.KT;
+}
+
+template <bool A_MK, bool B_KN>
+__global__ void __launch_bounds__(NT3, 1)
+    zgemm_dmma_ws(const GemmDesc *__restrict__ descs, int n_desc, long long total) {
+  using Cfg = V3Cfg<A_MK, B_KN>;
+  constexpr int ST3 = Cfg::ST;
+  extern __shared__ __align__(128) double2 smem[];
+  uint64_t *bars = reinterpret_cast<uint64_t *>(smem + ST3 * Cfg::STAGE);  // full[ST3], empty[ST3]
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+
+  const long long per = total / gridDim.x, rem = total % gridDim.x;
+  const long long t_begin = blockIdx.x * per + min((long long)blockIdx.x, rem);
+  const long long t_end = t_begin + per + ((long long)blockIdx.x < rem ? 1 : 0);
+  if (t_begin >= t_end) return;
+  int task = 0;
+  {
+    int lo = 0, hi = n_desc - 1;
+    while (lo < hi) {
+      int mid = (lo + hi + 1) >> 1;
+      if (descs[mid].tile_begin <= t_begin) lo = mid; else hi = mid - 1;
+    }
+    task = lo;
+  }
+  if (tid == 0) {
+    for (int s = 0; s < ST3; ++s) {
+      mbar_init(smem_u32(&bars[s]), 1);
+      mbar_init(smem_u32(&bars[ST3 + s]), NCW);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
+  }
+  __syncthreads();
+
+  if (warp == NCW) {
+    // ------------------------------------------------------------ producer warp
+    int step = 0;
+    for (long long tile = t_begin; tile < t_end; ++tile) {
+      V3Tile T;
+      v3_decode(descs, n_desc, task, tile, T);
+      const GemmDesc &d = *T.d;
+      const int Mi = d.Mi, Ni = d.Ni, Ki = d.Ki;
+      const double2 *Ab = d.A + T.t * d.sAt + T.mo * d.sAmo + (long long)T.m0 * d.sAmi;
+      const double2 *Bb = d.B + T.t * d.sBt + T.no * d.sBno + (long long)T.n0 * d.sBni;
+      const int mv = min(BM, Mi - T.m0), nv = min(BN, Ni - T.n0);  // valid rows / cols
+      for (int kt = 0; kt < T.KTOT; ++kt, ++step) {
+        const int slot = step % ST3;
+        const uint32_t full = smem_u32(&bars[slot]), empty = smem_u32(&bars[ST3 + slot]);
+        mbar_wait(empty, ((step / ST3) & 1) ^ 1);
+        const int ko = kt / T.KT;
+        const int kb = (kt - ko * T.KT) * BK2;
+        const int kv = min(BK2, Ki - kb);                          // valid k in this step
+        const double2 *Ak = Ab + ko * d.sAko + (long long)kb * d.sAki;
+        const double2 *Bk = Bb + ko * d.sBko + (long long)kb * d.sBki;
+        double2 *as = smem + slot * Cfg::STAGE;
+        double2 *bs = as + Cfg::A_ELEMS;
+        // rows of contiguous complex runs: A [m][k]: mv rows of kv; A [k][m]: kv rows of mv
+        const int a_rows = A_MK ? mv : kv, a_len = A_MK ? kv : mv, a_rows_all = A_MK ? BM : BK2;
+        const int a_full = A_MK ? BK2 : BM, a_pitch = A_MK ? PITCH_MK : PITCH_KM;
+        const long long a_rs = A_MK ? d.sAmi : d.sAki;
+        const int b_rows = B_KN ? kv : nv, b_len = B_KN ? nv : kv, b_rows_all = B_KN ? BK2 : BN;
+        const int b_full = B_KN ? BN : BK2, b_pitch = B_KN ? PITCH_KM : PITCH_MK;
+        const long long b_rs = B_KN ? d.sBki : d.sBni;
+        // zero-fill what the copies will not cover (ragged tiles only)
+        bool zf = false;
+        if (a_rows < a_rows_all || a_len < a_full) {
+          for (int i = lane; i < a_rows_all * a_full; i += 32) {
+            const int r = i / a_full, cidx = i - r * a_full;
+            if (r >= a_rows || cidx >= a_len) as[r * a_pitch + cidx] = make_double2(0.0, 0.0);
+          }
+          zf = true;
+        }
+        if (b_rows < b_rows_all || b_len < b_full) {
+          for (int i = lane; i < b_rows_all * b_full; i += 32) {
+            const int r = i / b_full, cidx = i - r * b_full;
+            if (r >= b_rows || cidx >= b_len) bs[r * b_pitch + cidx] = make_double2(0.0, 0.0);
+          }
+          zf = true;
+        }
+        if (zf) asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");
+        __syncwarp();
+        if (lane == 0) mbar_arrive_tx(full, (uint32_t)((a_rows * a_len + b_rows * b_len) * 16));
+        __syncwarp();
+        for (int r = lane; r < a_rows; r += 32)
+          bulk_g2s(smem_u32(as + r * a_pitch), Ak + r * a_rs, (uint32_t)(a_len * 16), full);
+        for (int r = lane; r < b_rows; r += 32)
+          bulk_g2s(smem_u32(bs + r * b_pitch), Bk + r * b_rs, (uint32_t)(b_len * 16), full);
+      }
+    }
+    return;
+  }
+
+  // -------------------------------------------------------------- consumer warps
+  // One consumer warp per SMSP: it must issue a DMMA every 16 cycles, so its shared-memory
+  // fragment loads for k-quad q+1 are issued before the DMMAs of q (double-buffered
+  // fragments), and the next stage is awaited one k-quad early.
+  const int wm = warp >> 1, wn = warp & 1;
+  double cr[4][4][2], ci[4][4][2];
+#pragma unroll
+  for (int i = 0; i < 4; ++i)
+#pragma unroll
+    for (int j = 0; j < 4; ++j) { cr[i][j][0] = cr[i][j][1] = ci[i][j][0] = ci[i][j][1] = 0.0; }
+  double fa[2][4][2], fb[2][4][2];  // [buffer][i or j][re, im]
+  auto load_frags = [&](int buf, const double2 *as, const double2 *bs, int kq) {
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      const int m = wm * 32 + i * 8 + (lane >> 2), k = kq * 4 + (lane & 3);
+      const double2 a = A_MK ? as[m * PITCH_MK + k] : as[k * PITCH_KM + m];
+      fa[buf][i][0] = a.x; fa[buf][i][1] = a.y;
+    }
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const int n = wn * 32 + j * 8 + (lane >> 2), k = kq * 4 + (lane & 3);
+      const double2 b = B_KN ? bs[k * PITCH_KM + n] : bs[n * PITCH_MK + k];
+      fb[buf][j][0] = b.x; fb[buf][j][1] = b.y;
+    }
+  };
+  auto mma_quad = [&](int buf) {
+#pragma unroll
+    for (int i = 0; i < 4; ++i)
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        dmma(cr[i][j][0], cr[i][j][1], fa[buf][i][0], fb[buf][j][0]);
+        dmma(ci[i][j][0], ci[i][j][1], fa[buf][i][0], fb[buf][j][1]);
+      }
+#pragma unroll
+    for (int i = 0; i < 4; ++i)
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        dmma(cr[i][j][0], cr[i][j][1], dneg(fa[buf][i][1]), fb[buf][j][1]);
+        dmma(ci[i][j][0], ci[i][j][1], fa[buf][i][1], fb[buf][j][0]);
+      }
+  };
+  // the whole CTA range is one sequence of k-steps; count them
+  int step = 0;
+  V3Tile T;
+  long long tile = t_begin;
+  v3_decode(descs, n_desc, task, tile, T);
+  int kt = 0;
+  mbar_wait(smem_u32(&bars[0]), 0);
+  load_frags(0, smem, smem + Cfg::A_ELEMS, 0);
+  for (;;) {
+    const int slot = step % ST3;
+    const double2 *as = smem + slot * Cfg::STAGE;
+    const double2 *bs = as + Cfg::A_ELEMS;
+    // is there a next k-step (this tile or the next)?
+    const bool last_k = (kt + 1 == T.KTOT);
+    const bool has_next = !last_k || (tile + 1 < t_end);
+    const int nslot = (slot + 1 == ST3) ? 0 : slot + 1;
+    const double2 *nas = smem + nslot * Cfg::STAGE;
+#pragma unroll
+    for (int kq = 0; kq < BK2 / 4; ++kq) {
+      const int cur = kq & 1;
+      if (kq + 1 < BK2 / 4) {
+        load_frags(cur ^ 1, as, bs, kq + 1);
+      } else if (has_next) {
+        mbar_wait(smem_u32(&bars[nslot]), ((step + 1) / ST3) & 1);
+        load_frags(cur ^ 1, nas, nas + Cfg::A_ELEMS, 0);
+      }
+      if (kq + 1 == BK2 / 4) {  // every fragment of this stage is in registers: release it
+        __syncwarp();
+        if (lane == 0) mbar_arrive(smem_u32(&bars[ST3 + slot]));
+      }
+      mma_quad(cur);
+    }
+    ++step;
+    if (!last_k) { ++kt; continue; }
+    // tile done: epilogue from registers (the producer keeps filling the next stages)
+    {
+      const GemmDesc &d = *T.d;
+      double2 *C = d.C + T.t * d.sCt + T.mo * d.sCmo + T.no * d.sCno;
+      const long long sCmi = d.sCmi, sCni = d.sCni;
+      const int Mi = d.Mi, Ni = d.Ni;
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {
+        const int m = T.m0 + wm * 32 + i * 8 + (lane >> 2);
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+          const int n = T.n0 + wn * 32 + j * 8 + (lane & 3) * 2;
+          if (m < Mi) {
+            double2 *cp = C + (long long)m * sCmi + (long long)n * sCni;
+            if (n < Ni) cp[0] = make_double2(cr[i][j][0], ci[i][j][0]);
+            if (n + 1 < Ni) cp[sCni] = make_double2(cr[i][j][1], ci[i][j][1]);
+          }
+          cr[i][j][0] = cr[i][j][1] = ci[i][j][0] = ci[i][j][1] = 0.0;
+        }
+      }
+    }
+    if (++tile >= t_end) break;
+    v3_decode(descs, n_desc, task, tile, T);
+    kt = 0;
+  }
+}
+
 // ---------------------------------------------------------------- dot / trace
 
 constexpr int DT = 256;
@@ -515,12 +789,37 @@ __global__ void accumulate_kernel(double2 *dst, const double2 *src, long long n)
 
 }  // namespace
 
-cudaError_t launch_gemm_group(const GemmDesc *d_descs, int n, long long total_tiles, cudaStream_t st) {
+int gemm_layout_class(const GemmDesc &d) {
+  const bool a_mk = d.sAki == 1 || d.Ki == 1, a_km = d.sAmi == 1 || d.Mi == 1;
+  const bool b_kn = d.sBni == 1 || d.Ni == 1, b_nk = d.sBki == 1 || d.Ki == 1;
+  if (!(a_mk || a_km) || !(b_kn || b_nk)) return 4;
+  return (a_mk ? 0 : 2) + (b_kn ? 0 : 1);
+}
+
+namespace {
+template <bool A_MK, bool B_KN>
+cudaError_t launch_ws(const GemmDesc *d_descs, int n, long long total, int sms, cudaStream_t st) {
+  using Cfg = V3Cfg<A_MK, B_KN>;
+  static bool attr = false;
+  if (!attr) {
+    cudaError_t e = cudaFuncSetAttribute(zgemm_dmma_ws<A_MK, B_KN>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         Cfg::SMEM);
+    if (e != cudaSuccess) return e;
+    attr = true;
+  }
+  long long grid = sms;  // one CTA (4 DMMA warps + 1 producer) per SM
+  if (grid > total) grid = total;
+  zgemm_dmma_ws<A_MK, B_KN><<<(unsigned)grid, NT3, Cfg::SMEM, st>>>(d_descs, n, total);
+  return cudaGetLastError();
+}
+}  // namespace
+
+cudaError_t launch_gemm_group(const GemmDesc *d_descs, int n, long long total_tiles, int cls, cudaStream_t st) {
   static bool attr_set = false;  // per process; the attribute is per-function, all devices
-  static int use_v1 = -1;
-  if (use_v1 < 0) {
-    const char *e = getenv("MICCO_GEMM_V1");
-    use_v1 = (e && e[0] == '1') ? 1 : 0;
+  static int variant = -1;       // MICCO_GEMM = 1 (per-tile), 2 (persistent cp.async), 3 (default: ws)
+  if (variant < 0) {
+    const char *e = getenv("MICCO_GEMM");
+    variant = (e && (e[0] == '1' || e[0] == '2')) ? e[0] - '0' : 3;
   }
   if (!attr_set) {
     cudaError_t e = cudaFuncSetAttribute(zgemm_dmma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, GEMM_SMEM);
@@ -530,18 +829,26 @@ cudaError_t launch_gemm_group(const GemmDesc *d_descs, int n, long long total_ti
     attr_set = true;
   }
   if (total_tiles <= 0) return cudaSuccess;
-  if (use_v1) {
+  int dev = 0, sms = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  if (variant == 1 || cls == 4) {
     long long grid = total_tiles < (1LL << 30) ? total_tiles : (1LL << 30);
     zgemm_dmma_kernel<<<(unsigned)grid, NT, GEMM_SMEM, st>>>(d_descs, n, total_tiles);
     return cudaGetLastError();
   }
-  int dev = 0, sms = 148;
-  cudaGetDevice(&dev);
-  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-  long long grid = 2LL * sms;  // 2 resident CTAs per SM (248 registers, 112 KB smem each)
-  if (grid > total_tiles) grid = total_tiles;
-  zgemm_dmma_persistent<<<(unsigned)grid, NT, GEMM2_SMEM, st>>>(d_descs, n, total_tiles);
-  return cudaGetLastError();
+  if (variant == 2) {
+    long long grid = 2LL * sms;  // 2 resident CTAs per SM (255 registers, 112 KB smem each)
+    if (grid > total_tiles) grid = total_tiles;
+    zgemm_dmma_persistent<<<(unsigned)grid, NT, GEMM2_SMEM, st>>>(d_descs, n, total_tiles);
+    return cudaGetLastError();
+  }
+  switch (cls) {
+    case 0: return launch_ws<true, true>(d_descs, n, total_tiles, sms, st);
+    case 1: return launch_ws<true, false>(d_descs, n, total_tiles, sms, st);
+    case 2: return launch_ws<false, true>(d_descs, n, total_tiles, sms, st);
+    default: return launch_ws<false, false>(d_descs, n, total_tiles, sms, st);
+  }
 }
 
 cudaError_t launch_dot_group(const DotDesc *d_descs, int n, long long total_ctas, cudaStream_t st) {

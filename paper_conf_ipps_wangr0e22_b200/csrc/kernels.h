@@ -24,7 +24,7 @@ struct GemmDesc {
   long long sAmo, sAmi, sAko, sAki;
   long long sBko, sBki, sBno, sBni;
   long long sCmo, sCmi, sCno, sCni;
-  int Lt, tilesM, tilesN, pad;
+  int Lt, tilesM, tilesN, cls;  // cls: operand layout class (gemm_layout_class)
   long long tile_begin;  // first CTA tile of this task in the grouped launch
 };
 
@@ -49,8 +49,14 @@ struct DotDesc {
 
 constexpr int kGemmBM = 64, kGemmBN = 64, kGemmBK = 8, kGemmStages = 4, kGemmThreads = 128;
 
-// Grouped launches: descs in device memory; grid covers total tiles / CTAs.
-cudaError_t launch_gemm_group(const GemmDesc *d_descs, int n, long long total_tiles, cudaStream_t st);
+// Layout class of a GEMM descriptor: 0 = A[m][k] B[k][n], 1 = A[m][k] B[n][k],
+// 2 = A[k][m] B[k][n], 3 = A[k][m] B[n][k] (unit-stride inner index of each operand),
+// 4 = some operand has no unit-stride inner index (generic gather kernel).
+int gemm_layout_class(const GemmDesc &d);
+constexpr int kGemmClasses = 5;
+
+// Grouped launches: descs in device memory (all of one layout class); grid covers the tiles.
+cudaError_t launch_gemm_group(const GemmDesc *d_descs, int n, long long total_tiles, int cls, cudaStream_t st);
 cudaError_t launch_dot_group(const DotDesc *d_descs, int n, long long total_ctas, cudaStream_t st);
 
 // vals[g][t] = Π_{c in comps(g)} S[slot_c][t] (component scalars)
