@@ -493,7 +493,7 @@ __global__ void __launch_bounds__(NT3, 1)
   }
   if (tid == 0) {
     for (int s = 0; s < ST3; ++s) {
-      mbar_init(smem_u32(&bars[s]), 1);
+      mbar_init(smem_u32(&bars[s]), 32);
       mbar_init(smem_u32(&bars[ST3 + s]), NCW);
     }
     asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
@@ -502,59 +502,53 @@ __global__ void __launch_bounds__(NT3, 1)
 
   if (warp == NCW) {
     // ------------------------------------------------------------ producer warp
+    // Per-thread 16-byte cp.async (LDGSTS) along the unit-stride index of each operand (the
+    // bulk-copy variant serialised one UBLKCP per row through the uniform datapath and could
+    // not keep up), zero-fill by src-size 0 for ragged rows/tails, and completion signalled
+    // to the stage's "full" mbarrier by cp.async.mbarrier.arrive.noinc from every lane.
     int step = 0;
     for (long long tile = t_begin; tile < t_end; ++tile) {
       V3Tile T;
       v3_decode(descs, n_desc, task, tile, T);
       const GemmDesc &d = *T.d;
-      const int Mi = d.Mi, Ni = d.Ni, Ki = d.Ki;
-      const double2 *Ab = d.A + T.t * d.sAt + T.mo * d.sAmo + (long long)T.m0 * d.sAmi;
-      const double2 *Bb = d.B + T.t * d.sBt + T.no * d.sBno + (long long)T.n0 * d.sBni;
-      const int mv = min(BM, Mi - T.m0), nv = min(BN, Ni - T.n0);  // valid rows / cols
+      const int Ki = d.Ki;
+      const long long sAmi = d.sAmi, sAki = d.sAki, sBki = d.sBki, sBni = d.sBni;
+      const double2 *Ab = d.A + T.t * d.sAt + T.mo * d.sAmo + (long long)T.m0 * sAmi;
+      const double2 *Bb = d.B + T.t * d.sBt + T.no * d.sBno + (long long)T.n0 * sBni;
+      const int mv = min(BM, d.Mi - T.m0), nv = min(BN, d.Ni - T.n0);  // valid rows / cols
       for (int kt = 0; kt < T.KTOT; ++kt, ++step) {
         const int slot = step % ST3;
         const uint32_t full = smem_u32(&bars[slot]), empty = smem_u32(&bars[ST3 + slot]);
         mbar_wait(empty, ((step / ST3) & 1) ^ 1);
         const int ko = kt / T.KT;
         const int kb = (kt - ko * T.KT) * BK2;
-        const int kv = min(BK2, Ki - kb);                          // valid k in this step
-        const double2 *Ak = Ab + ko * d.sAko + (long long)kb * d.sAki;
-        const double2 *Bk = Bb + ko * d.sBko + (long long)kb * d.sBki;
+        const int kv = min(BK2, Ki - kb);  // valid k in this step
+        const double2 *Ak = Ab + ko * d.sAko + (long long)kb * sAki;
+        const double2 *Bk = Bb + ko * d.sBko + (long long)kb * sBki;
         double2 *as = smem + slot * Cfg::STAGE;
         double2 *bs = as + Cfg::A_ELEMS;
-        // rows of contiguous complex runs: A [m][k]: mv rows of kv; A [k][m]: kv rows of mv
-        const int a_rows = A_MK ? mv : kv, a_len = A_MK ? kv : mv, a_rows_all = A_MK ? BM : BK2;
-        const int a_full = A_MK ? BK2 : BM, a_pitch = A_MK ? PITCH_MK : PITCH_KM;
-        const long long a_rs = A_MK ? d.sAmi : d.sAki;
-        const int b_rows = B_KN ? kv : nv, b_len = B_KN ? nv : kv, b_rows_all = B_KN ? BK2 : BN;
-        const int b_full = B_KN ? BN : BK2, b_pitch = B_KN ? PITCH_KM : PITCH_MK;
-        const long long b_rs = B_KN ? d.sBki : d.sBni;
-        // zero-fill what the copies will not cover (ragged tiles only)
-        bool zf = false;
-        if (a_rows < a_rows_all || a_len < a_full) {
-          for (int i = lane; i < a_rows_all * a_full; i += 32) {
-            const int r = i / a_full, cidx = i - r * a_full;
-            if (r >= a_rows || cidx >= a_len) as[r * a_pitch + cidx] = make_double2(0.0, 0.0);
-          }
-          zf = true;
+#pragma unroll 4
+        for (int j = 0; j < (BM * BK2) / 32; ++j) {
+          const int e = lane + 32 * j;
+          int m, k;
+          if (A_MK) { k = e & (BK2 - 1); m = e / BK2; } else { m = e & (BM - 1); k = e / BM; }
+          const bool v = m < mv && k < kv;
+          const double2 *src = v ? Ak + m * sAmi + k * sAki : d.A;
+          cp_async16(A_MK ? as + m * PITCH_MK + k : as + k * PITCH_KM + m, src, v);
         }
-        if (b_rows < b_rows_all || b_len < b_full) {
-          for (int i = lane; i < b_rows_all * b_full; i += 32) {
-            const int r = i / b_full, cidx = i - r * b_full;
-            if (r >= b_rows || cidx >= b_len) bs[r * b_pitch + cidx] = make_double2(0.0, 0.0);
-          }
-          zf = true;
+#pragma unroll 4
+        for (int j = 0; j < (BN * BK2) / 32; ++j) {
+          const int e = lane + 32 * j;
+          int n, k;
+          if (B_KN) { n = e & (BN - 1); k = e / BN; } else { k = e & (BK2 - 1); n = e / BK2; }
+          const bool v = n < nv && k < kv;
+          const double2 *src = v ? Bk + k * sBki + n * sBni : d.B;
+          cp_async16(B_KN ? bs + k * PITCH_KM + n : bs + n * PITCH_MK + k, src, v);
         }
-        if (zf) asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");
-        __syncwarp();
-        if (lane == 0) mbar_arrive_tx(full, (uint32_t)((a_rows * a_len + b_rows * b_len) * 16));
-        __syncwarp();
-        for (int r = lane; r < a_rows; r += 32)
-          bulk_g2s(smem_u32(as + r * a_pitch), Ak + r * a_rs, (uint32_t)(a_len * 16), full);
-        for (int r = lane; r < b_rows; r += 32)
-          bulk_g2s(smem_u32(bs + r * b_pitch), Bk + r * b_rs, (uint32_t)(b_len * 16), full);
+        asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];\n" ::"r"(full) : "memory");
       }
     }
+    asm volatile("cp.async.wait_all;\n" ::: "memory");
     return;
   }
 
