@@ -178,6 +178,8 @@ struct Plan {
   double flops = 0, max_over_mean_load = 1, predicted_s = 0;
   std::vector<double> gpu_flops;
   std::vector<std::pair<int32_t, uint64_t>> final_nodes;  // (node tensor, GPU mask) left cached
+  std::vector<int32_t> fused_dot;  // GEMM task → DOT task fused into its epilogue, or -1
+  int64_t n_fused = 0;
 };
 
 struct PlanInput {
@@ -187,6 +189,7 @@ struct PlanInput {
   std::vector<int64_t> budget;                      // per GPU
   int32_t window_graphs;
   bool keep_inputs;
+  bool fuse = true;                                 // fuse GEMM → final dot when legal
   std::vector<std::vector<int32_t>> initial_nodes;  // per GPU: node tensors already resident
   double peer_gbs, host_gbs, flops_per_s;           // cost model of the bound sweep
 };

@@ -20,6 +20,7 @@
 
 #include <algorithm>
 #include <chrono>
+#include <cstdlib>
 #include <cstring>
 #include <string>
 #include <unordered_map>
@@ -143,6 +144,7 @@ struct LGpu {
   std::unordered_map<int32_t, std::vector<cudaEvent_t>> readers;  // peer reads to wait for before free
   std::vector<GemmDesc> gemm;
   std::vector<DotDesc> dot;
+  std::vector<double2 *> part_allocs;  // fused-dot partials of the pending batch
   long long gemm_tiles = 0, dot_ctas = 0;
   char *ring_h = nullptr, *ring_d = nullptr;
   cudaEvent_t ring_ev[kRingSlots] = {};
@@ -167,6 +169,7 @@ struct Executor::Impl {
   std::vector<int64_t> budget_cache;
   int budget_cache_n = 0;
   std::vector<std::pair<int32_t, uint64_t>> cached_nodes;
+  std::vector<int32_t> fused_dot;  // of the plan being replayed
   int32_t chosen_bd[3] = {0, 0, 0};
   int chosen_bd_n = 0;
   // results on device 0
@@ -389,6 +392,8 @@ struct Executor::Impl {
       }
       return acc;
     });
+    for (double2 *p : l.part_allocs) CK(cudaFreeAsync(p, l.st));
+    l.part_allocs.clear();
   }
 
   void compute(LGpu &l, int32_t task, micco_stats &st) {
@@ -406,7 +411,8 @@ struct Executor::Impl {
       const long long lim = (1LL << 31) - 1;  // the GEMM keeps per-slice offsets in 32 bits
       if (L.sliceA > lim || L.sliceB > lim || L.sliceC > lim)
         fail(MICCO_ERR_UNSUPPORTED, "executor: tensor slice exceeds 2^31 elements");
-      double2 *pc = alloc(l, bytes_of(tk.out));
+      const int32_t fd = fused_dot.empty() ? -1 : fused_dot[task];
+      double2 *pc = fd >= 0 ? nullptr : alloc(l, bytes_of(tk.out));
       l.ptr[tk.out] = pc;
       GemmDesc d{};
       d.A = pa; d.B = pb; d.C = pc;
@@ -418,7 +424,33 @@ struct Executor::Impl {
       d.Lt = c.Lt;
       d.tilesM = (L.Mi + kGemmBM - 1) / kGemmBM;
       d.tilesN = (L.Ni + kGemmBN - 1) / kGemmBN;
-      d.cls = gemm_layout_class(d);
+      d.cls = gemm_class(L);
+      if (fd >= 0) {  // final dot in the epilogue: C is never materialised
+        const TaskRec &dk = c.tasks[fd];
+        const int32_t X = tk.out, Y = dk.a == X ? dk.b : dk.a;
+        const TensorRec &YT = c.tensors[Y];
+        int q[2] = {0, 1};  // Y leg paired with X leg 0 (M) and X leg 1 (N)
+        for (int i = 0; i < dk.c; ++i) {
+          if (dk.a == X) q[dk.pa[i]] = dk.pb[i]; else q[dk.pb[i]] = dk.pa[i];
+        }
+        const long long sY[2] = {YT.dim[1], 1};
+        d.D = l.ptr[Y];
+        if (!d.D) fail(MICCO_ERR_STATE, "executor: fused dot partner not resident");
+        d.sDt = YT.slice_elems;
+        d.sDmo = d.sDno = 0;
+        d.sDmi = sY[q[0]];
+        d.sDni = sY[q[1]];
+        const long long tps = (long long)L.Mo * L.No * d.tilesM * d.tilesN * 4;  // partials per slice
+        d.part = alloc(l, tps * c.Lt * 16);
+        l.part_allocs.push_back(d.part);
+        DotDesc r{};
+        r.A = d.part; r.B = nullptr;
+        r.out = devs[l.dev].scalars + (size_t)c.tensors[dk.out].scalar_slot * c.Lt;
+        r.sAt = tps; r.mode = 3; r.X = (int)tps; r.Lt = c.Lt;
+        for (int i = 0; i < 3; ++i) r.O[i] = 1;
+        l.dot.push_back(r);
+        st.dot_bytes += (double)YT.slice_elems * 16.0 * c.Lt;
+      }
       l.gemm.push_back(d);
       st.gemm_flops += tk.flops;
     } else {
@@ -561,6 +593,10 @@ struct Executor::Impl {
     in.budget = budgets();
     in.window_graphs = c.opt.window_graphs;
     in.keep_inputs = c.opt.keep_inputs_resident != 0;
+    {
+      const char *gv = getenv("MICCO_GEMM"), *nf = getenv("MICCO_NO_FUSE");
+      in.fuse = !(gv && (gv[0] == '1' || gv[0] == '2')) && !(nf && nf[0] == '1');
+    }
     in.peer_gbs = (ndev > 1 && !dist()) || dist() ? 700 : 2500;
     in.host_gbs = 55;
     in.flops_per_s = 30e12;
@@ -587,6 +623,7 @@ struct Executor::Impl {
       chosen_bd_n = n;
     }
     cached_nodes = plan.final_nodes;
+    fused_dot = plan.fused_dot;
     auto t1 = std::chrono::steady_clock::now();
 
     micco_stats st{};

@@ -26,6 +26,13 @@ struct GemmDesc {
   long long sCmo, sCmi, sCno, sCni;
   int Lt, tilesM, tilesN, cls;  // cls: operand layout class (gemm_layout_class)
   long long tile_begin;  // first CTA tile of this task in the grouped launch
+  // Fused final contraction (GEMM → dot, SURVEY.md §8(a) A9 "fused into the last GEMM's
+  // epilogue"): when D != nullptr, C is never written; instead every consumer warp writes
+  //   part[(task tile) * 4 + warp] = Σ_{its (m, n)} C[t][m][n] · D[t][m·sD_m + n·sD_n]
+  // and a fixed-order partial sum (zdot mode 3) produces the scalar per slice.
+  const double2 *D;
+  double2 *part;
+  long long sDt, sDmo, sDmi, sDno, sDni;
 };
 
 // The final reduction of two nodes to a scalar per slice ("until
@@ -34,6 +41,7 @@ struct GemmDesc {
 //   mode 0: x is contiguous in both A and B (flat run of X elements per outer index)
 //   mode 1: x contiguous in A, y contiguous in B → 32×32 shared-memory transpose tiles
 //   mode 2: trace (stride sAx along x)
+//   mode 3: Σ_x A[x] (fixed-order sum of X partials of a fused GEMM → dot)
 struct DotDesc {
   const double2 *A;
   const double2 *B;
@@ -49,10 +57,8 @@ struct DotDesc {
 
 constexpr int kGemmBM = 64, kGemmBN = 64, kGemmBK = 8, kGemmStages = 4, kGemmThreads = 128;
 
-// Layout class of a GEMM descriptor: 0 = A[m][k] B[k][n], 1 = A[m][k] B[n][k],
-// 2 = A[k][m] B[k][n], 3 = A[k][m] B[n][k] (unit-stride inner index of each operand),
-// 4 = some operand has no unit-stride inner index (generic gather kernel).
-int gemm_layout_class(const GemmDesc &d);
+// GEMM descriptors carry their operand-layout class (layout.h gemm_class): 0..3 = unit-stride
+// inner index for both operands (warp-specialized kernel), 4 = generic gather kernel.
 constexpr int kGemmClasses = 5;
 
 // Grouped launches: descs in device memory (all of one layout class); grid covers the tiles.

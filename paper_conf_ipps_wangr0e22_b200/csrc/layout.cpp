@@ -95,6 +95,13 @@ bool gemm_layout(int ra, const int32_t *dA, int rb, const int32_t *dB, int c, co
   return true;
 }
 
+int gemm_class(const GemmLayout &L) {
+  const bool a_mk = L.sAki == 1 || L.Ki == 1, a_km = L.sAmi == 1 || L.Mi == 1;
+  const bool b_kn = L.sBni == 1 || L.Ni == 1, b_nk = L.sBki == 1 || L.Ki == 1;
+  if (!(a_mk || a_km) || !(b_kn || b_nk)) return 4;
+  return (a_mk ? 0 : 2) + (b_kn ? 0 : 1);
+}
+
 bool dot_layout(int ra, const int32_t *dA, int rb, const int32_t *dB, int c, const int8_t *pa,
                 const int8_t *pb, DotLayout &L) {
   long long sA[8], sB[8];

@@ -29,6 +29,10 @@ struct DotLayout {
 bool gemm_layout(int ra, const int32_t *dA, int rb, const int32_t *dB, int c, const int8_t *pa,
                  const int8_t *pb, GemmLayout &L);
 
+// operand-layout class of the GEMM kernels (kernels.h): 0 A[m][k] B[k][n], 1 A[m][k] B[n][k],
+// 2 A[k][m] B[k][n], 3 A[k][m] B[n][k], 4 = an operand without a unit-stride inner index
+int gemm_class(const GemmLayout &L);
+
 // full contraction of A with B (rank r each, pairs (pa[i], pb[i])), or a meson trace
 // (B absent: rb = 0).  false = unsupported.
 bool dot_layout(int ra, const int32_t *dA, int rb, const int32_t *dB, int c, const int8_t *pa,

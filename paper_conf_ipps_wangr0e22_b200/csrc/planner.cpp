@@ -19,6 +19,7 @@
 #include <string>
 
 #include "core.h"
+#include "layout.h"
 #include "scheduler.h"
 
 namespace micco {
@@ -171,11 +172,55 @@ Plan make_plan(const Context &ctx, const PlanInput &in) {
       }
     }
   }
+  // 1b. fuse a final dot into the GEMM that produces its operand when that product X is a
+  // matrix used by nothing else and the dot's other operand Y exists before the GEMM's
+  // stage: X is never written, Y is read in the GEMM epilogue (kernels.h GemmDesc::D).
+  // Decided from the DAG alone, so it is identical for every GPU count.
+  plan.fused_dot.assign(T, -1);
+  std::vector<char> skip(T, 0);
+  std::vector<int32_t> extra(T, -1);  // fused GEMM task → Y
+  if (in.fuse) {
+    std::vector<int32_t> consumers(NT, 0);
+    for (int32_t t = 0; t < T; ++t) {
+      const TaskRec &tk = ctx.tasks[t];
+      if (tk.a >= 0) ++consumers[tk.a];
+      if (tk.b >= 0 && tk.b != tk.a) ++consumers[tk.b];
+    }
+    for (int32_t d = 0; d < T; ++d) {
+      const TaskRec &dk = ctx.tasks[d];
+      if (dk.kind != TASK_DOT || dk.a == dk.b || task_window[d] < 0) continue;
+      for (int side = 0; side < 2; ++side) {
+        const int32_t X = side == 0 ? dk.a : dk.b, Y = side == 0 ? dk.b : dk.a;
+        const int32_t pt = ctx.tensors[X].task;
+        if (pt < 0 || consumers[X] != 1 || ctx.tensors[X].rank != 2) continue;
+        const TaskRec &pk = ctx.tasks[pt];
+        if (pk.kind != TASK_GEMM || plan.fused_dot[pt] >= 0 || ctx.tensors[Y].level >= pk.level) continue;
+        const TensorRec &A = ctx.tensors[pk.a], &B = ctx.tensors[pk.b];
+        if (A.rank - pk.c != 1 || B.rank - pk.c != 1) continue;  // one M leg, one N leg
+        GemmLayout L;
+        if (!gemm_layout(A.rank, A.dim, B.rank, B.dim, pk.c, pk.pa, pk.pb, L) || gemm_class(L) == 4) continue;
+        plan.fused_dot[pt] = d;
+        extra[pt] = Y;
+        skip[d] = 1;
+        ++plan.n_fused;
+        break;
+      }
+    }
+  }
+  auto operands = [&](int32_t t, int32_t out[3]) {  // distinct tensors a task reads
+    const TaskRec &tk = ctx.tasks[t];
+    int k = 0;
+    out[k++] = tk.a;
+    if (tk.b >= 0 && tk.b != tk.a) out[k++] = tk.b;
+    if (extra[t] >= 0 && extra[t] != tk.a && extra[t] != tk.b) out[k++] = extra[t];
+    return k;
+  };
+
   // 2. stages = (window, level), tasks in id order inside a stage
   std::vector<int32_t> order;
   order.reserve(T);
   for (int32_t t = 0; t < T; ++t)
-    if (task_window[t] >= 0) order.push_back(t);
+    if (task_window[t] >= 0 && !skip[t]) order.push_back(t);
   std::stable_sort(order.begin(), order.end(), [&](int32_t x, int32_t y) {
     if (task_window[x] != task_window[y]) return task_window[x] < task_window[y];
     return ctx.tasks[x].level < ctx.tasks[y].level;
@@ -197,9 +242,10 @@ Plan make_plan(const Context &ctx, const PlanInput &in) {
   S.use_stages.assign(NT, {});
   for (int32_t s = 0; s < (int32_t)stages.size(); ++s)
     for (int32_t i = stages[s].first; i < stages[s].second; ++i) {
-      const TaskRec &tk = ctx.tasks[order[i]];
-      for (int32_t op : {tk.a, tk.b}) {
-        if (op < 0 || (op == tk.b && tk.b == tk.a)) continue;
+      int32_t ops[3];
+      const int k = operands(order[i], ops);
+      for (int j = 0; j < k; ++j) {
+        const int32_t op = ops[j];
         ++S.uses_left[op];
         if (S.use_stages[op].empty() || S.use_stages[op].back() != s) S.use_stages[op].push_back(s);
       }
@@ -240,14 +286,16 @@ Plan make_plan(const Context &ctx, const PlanInput &in) {
       const int32_t a = tk.a, b = tk.b;
       const bool same = (b < 0 || b == a);
       const TensorRec &out = ctx.tensors[tk.out];
+      const int32_t y = extra[t];  // fused dot partner (read in the epilogue), or -1
+      const bool has_y = y >= 0 && y != a && y != b;
       SchedPair p;
       p.m1 = S.mask[a];
       p.m2 = same ? S.mask[a] : S.mask[b];
       p.same = same;
       p.b1 = S.bytes(a);
       p.b2 = same ? 0 : S.bytes(b);
-      p.bout = out.rank > 0 ? S.bytes(tk.out) : 0;
-      p.flops = tk.flops;
+      p.bout = (out.rank > 0 && y < 0) ? S.bytes(tk.out) : 0;
+      p.flops = tk.flops + (y >= 0 ? ctx.tasks[plan.fused_dot[t]].flops : 0.0);
       sched.mem = S.mem;
       const int g = sched.decide(p);
       const uint64_t bit = 1ULL << g;
@@ -255,15 +303,18 @@ Plan make_plan(const Context &ctx, const PlanInput &in) {
         int64_t need = p.bout;
         if (!(S.mask[a] & bit)) need += p.b1;
         if (!same && !(S.mask[b] & bit)) need += p.b2;
+        if (has_y && !(S.mask[y] & bit)) need += S.bytes(y);
         return need;
       };
       // pin operands so the eviction below never drops them
       S.pin[g][a] = S.epoch[g];
       if (!same) S.pin[g][b] = S.epoch[g];
+      if (has_y) S.pin[g][y] = S.epoch[g];
       if (!S.make_room(g, need_bytes())) {
         flush(g);  // split the stage: run what is pinned, then retry with this pair only
         S.pin[g][a] = S.epoch[g];
         if (!same) S.pin[g][b] = S.epoch[g];
+        if (has_y) S.pin[g][y] = S.epoch[g];
         if (!S.make_room(g, need_bytes()))
           fail(MICCO_ERR_OOM, "planner: one contraction's operands and output (" +
                                   std::to_string(need_bytes()) + " B) exceed the GPU budget (" +
@@ -271,26 +322,27 @@ Plan make_plan(const Context &ctx, const PlanInput &in) {
       }
       if (S.mask[a] & bit) ++plan.cache_hits; else S.fetch(g, a);
       if (!same) { if (S.mask[b] & bit) ++plan.cache_hits; else S.fetch(g, b); }
-      if (out.rank > 0) {
+      if (has_y) { if (S.mask[y] & bit) ++plan.cache_hits; else S.fetch(g, y); }
+      if (out.rank > 0 && y < 0) {
         S.add_res(g, tk.out);
         S.pin[g][tk.out] = S.epoch[g];
       }
       sched.account(g, p);
       plan.task_gpu[t] = g;
-      plan.gpu_flops[g] += tk.flops;
-      plan.flops += tk.flops;
-      S.st_flops[g] += tk.flops;
+      if (y >= 0) plan.task_gpu[plan.fused_dot[t]] = g;
+      plan.gpu_flops[g] += p.flops;
+      plan.flops += p.flops;
+      S.st_flops[g] += p.flops;
       chunk[g].push_back(t);
     }
     for (int g = 0; g < n; ++g)
       if (!chunk[g].empty()) flush(g);
     // release operands whose last consumer ran
     for (int32_t i = stages[s].first; i < stages[s].second; ++i) {
-      const TaskRec &tk = ctx.tasks[order[i]];
-      for (int32_t op : {tk.a, tk.b}) {
-        if (op < 0 || (op == tk.b && tk.b == tk.a)) continue;
-        if (--S.uses_left[op] == 0) S.release(op);
-      }
+      int32_t ops[3];
+      const int k = operands(order[i], ops);
+      for (int j = 0; j < k; ++j)
+        if (--S.uses_left[ops[j]] == 0) S.release(ops[j]);
     }
     double worst = 0;
     for (int g = 0; g < n; ++g) {
