@@ -495,7 +495,11 @@ struct Executor::Impl {
         if (it != spill_ev.end() && c.tensors[op.id].node < 0) CK(cudaStreamWaitEvent(l.cst, it->second.second, 0));
         void *p = nullptr;
         CK(cudaMallocAsync(&p, (size_t)bytes_of(op.id), l.cst));
+        Timed tm{devs[l.dev].timing_events.get(), devs[l.dev].timing_events.get(), 2, l.dev};
+        CK(cudaEventRecord(tm.a, l.cst));
         CK(cudaMemcpyAsync(p, host_src(op.id), bytes_of(op.id), cudaMemcpyHostToDevice, l.cst));
+        CK(cudaEventRecord(tm.b, l.cst));
+        timed.push_back(tm);
         cudaEvent_t done = devs[l.dev].sync_events.get();
         CK(cudaEventRecord(done, l.cst));
         CK(cudaStreamWaitEvent(l.st, done, 0));
@@ -595,7 +599,7 @@ struct Executor::Impl {
     in.keep_inputs = c.opt.keep_inputs_resident != 0;
     {
       const char *gv = getenv("MICCO_GEMM"), *nf = getenv("MICCO_NO_FUSE");
-      in.fuse = !(gv && (gv[0] == '1' || gv[0] == '2')) && !(nf && nf[0] == '1');
+      in.fuse = gv && gv[0] == '3' && !(nf && nf[0] == '1');  // the fused epilogue exists in v3 only
     }
     in.peer_gbs = (ndev > 1 && !dist()) || dist() ? 700 : 2500;
     in.host_gbs = 55;
@@ -740,6 +744,7 @@ struct Executor::Impl {
       float ms = 0;
       CK(cudaSetDevice(tm.dev));
       CK(cudaEventElapsedTime(&ms, tm.a, tm.b));
+      if (tm.kind == 2) { st.copy_ms += ms; continue; }
       st.kernel_ms += ms;
       if (tm.kind == 0) { st.gemm_kernel_ms += ms; ++st.gemm_launches; }
       else if (tm.kind == 1) { st.dot_kernel_ms += ms; ++st.dot_launches; }

@@ -193,8 +193,8 @@ constexpr int BPITCH2 = BN + 2;   // 1056 B ≡ 32 (mod 128)
 constexpr int A_STAGE2 = BM * APITCH2;
 constexpr int B_STAGE2 = BK2 * BPITCH2;
 constexpr int GEMM2_SMEM = ST2 * (A_STAGE2 + B_STAGE2) * 16;
-constexpr int LPT = (BM * BK2) / NT;  // elements per thread per operand per stage (8)
 
+template <int LPT>
 struct LoadCur {
   const double2 *A, *B;  // tile bases (t, mo/no, m0/n0 applied)
   long long sAko, sBko;
@@ -210,8 +210,9 @@ struct StoreCur {
   int sCmi, sCni, Mi, Ni, m0, n0, KTOT;
 };
 
+template <int NTH, int LPT>
 __device__ __forceinline__ void decode_tile(const GemmDesc *__restrict__ descs, int n_desc, int &task,
-                                            long long tile, int tid, LoadCur *L, StoreCur *S) {
+                                            long long tile, int tid, LoadCur<LPT> *L, StoreCur *S) {
   while (task + 1 < n_desc && descs[task + 1].tile_begin <= tile) ++task;
   const GemmDesc &d = descs[task];
   long long lt = tile - d.tile_begin;
@@ -235,7 +236,7 @@ __device__ __forceinline__ void decode_tile(const GemmDesc *__restrict__ descs, 
     L->vA = 0; L->vB = 0;
 #pragma unroll
     for (int j = 0; j < LPT; ++j) {
-      const int e = tid + j * NT;
+      const int e = tid + j * NTH;
       int m, k, n, kb;
       if (L->akf) { k = e & (BK2 - 1); m = e / BK2; } else { m = e & (BM - 1); k = e / BM; }
       L->offA[j] = m * sAmi + k * sAki;
@@ -253,13 +254,19 @@ __device__ __forceinline__ void decode_tile(const GemmDesc *__restrict__ descs, 
   }
 }
 
-__global__ void __launch_bounds__(NT, 2)
+// NWM × NWN warps; warp tile (64/NWM) × (64/NWN) complex.  <2,2> = 128 threads with 32×32
+// warp tiles (248-255 registers, 2 warps per SMSP); <2,4> = 256 threads with 32×16 warp
+// tiles (half the accumulators, 4 warps per SMSP for latency hiding).
+template <int NWM, int NWN>
+__global__ void __launch_bounds__(NWM * NWN * 32, 2)
     zgemm_dmma_persistent(const GemmDesc *__restrict__ descs, int n_desc, long long total) {
+  constexpr int NTH = NWM * NWN * 32, LPT = (BM * BK2) / NTH;
+  constexpr int MI = BM / NWM / 8, NJ = BN / NWN / 8;  // 8x8 blocks per warp
   extern __shared__ __align__(128) double2 smem[];
   double2 *As = smem;
   double2 *Bs = smem + ST2 * A_STAGE2;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  const int wm = warp >> 1, wn = warp & 1;
+  const int wm = warp / NWN, wn = warp % NWN;
 
   const long long per = total / gridDim.x, rem = total % gridDim.x;
   const long long t_begin = blockIdx.x * per + min((long long)blockIdx.x, rem);
@@ -275,12 +282,12 @@ __global__ void __launch_bounds__(NT, 2)
     }
     task_l = task_c = lo;
   }
-  LoadCur L;
+  LoadCur<LPT> L;
   StoreCur S;
   long long tile_l = t_begin, tile_c = t_begin;
   int kt_l = 0, kt_c = 0;
-  decode_tile(descs, n_desc, task_l, tile_l, tid, &L, nullptr);
-  decode_tile(descs, n_desc, task_c, tile_c, tid, nullptr, &S);
+  decode_tile<NTH, LPT>(descs, n_desc, task_l, tile_l, tid, &L, nullptr);
+  decode_tile<NTH, LPT>(descs, n_desc, task_c, tile_c, tid, (LoadCur<LPT> *)nullptr, &S);
   bool more_l = true;
 
   auto issue_load = [&](int slot) {
@@ -292,7 +299,7 @@ __global__ void __launch_bounds__(NT, 2)
     double2 *bs = Bs + slot * B_STAGE2;
 #pragma unroll
     for (int j = 0; j < LPT; ++j) {
-      const int e = tid + j * NT;
+      const int e = tid + j * NTH;
       int m, k;
       if (L.akf) { k = e & (BK2 - 1); m = e / BK2; } else { m = e & (BM - 1); k = e / BM; }
       const bool v = ((L.vA >> j) & 1u) && (kb + k < L.Ki);
@@ -300,7 +307,7 @@ __global__ void __launch_bounds__(NT, 2)
     }
 #pragma unroll
     for (int j = 0; j < LPT; ++j) {
-      const int e = tid + j * NT;
+      const int e = tid + j * NTH;
       int n, k;
       if (L.bnf) { n = e & (BN - 1); k = e / BN; } else { k = e & (BK2 - 1); n = e / BK2; }
       const bool v = ((L.vB >> j) & 1u) && (kb + k < L.Ki);
@@ -309,16 +316,16 @@ __global__ void __launch_bounds__(NT, 2)
     // advance the load cursor (possibly into the next tile)
     if (++kt_l == L.KTOT) {
       kt_l = 0;
-      if (++tile_l < t_end) decode_tile(descs, n_desc, task_l, tile_l, tid, &L, nullptr);
+      if (++tile_l < t_end) decode_tile<NTH, LPT>(descs, n_desc, task_l, tile_l, tid, &L, nullptr);
       else more_l = false;
     }
   };
 
-  double cr[4][4][2], ci[4][4][2];
+  double cr[MI][NJ][2], ci[MI][NJ][2];
 #pragma unroll
-  for (int i = 0; i < 4; ++i)
+  for (int i = 0; i < MI; ++i)
 #pragma unroll
-    for (int j = 0; j < 4; ++j) { cr[i][j][0] = cr[i][j][1] = ci[i][j][0] = ci[i][j][1] = 0.0; }
+    for (int j = 0; j < NJ; ++j) { cr[i][j][0] = cr[i][j][1] = ci[i][j][0] = ci[i][j][1] = 0.0; }
 
 #pragma unroll
   for (int s = 0; s < ST2 - 1; ++s) {
@@ -336,28 +343,28 @@ __global__ void __launch_bounds__(NT, 2)
     const double2 *bs = Bs + slot_c * B_STAGE2;
 #pragma unroll
     for (int kq = 0; kq < BK2 / 4; ++kq) {
-      double ar[4], ai[4], an[4], br[4], bi[4];
+      double ar[MI], ai[MI], an[MI], br[NJ], bi[NJ];
 #pragma unroll
-      for (int i = 0; i < 4; ++i) {
-        const double2 a = as[(wm * 32 + i * 8 + (lane >> 2)) * APITCH2 + kq * 4 + (lane & 3)];
+      for (int i = 0; i < MI; ++i) {
+        const double2 a = as[(wm * MI * 8 + i * 8 + (lane >> 2)) * APITCH2 + kq * 4 + (lane & 3)];
         ar[i] = a.x; ai[i] = a.y; an[i] = dneg(a.y);
       }
 #pragma unroll
-      for (int j = 0; j < 4; ++j) {
-        const double2 b = bs[(kq * 4 + (lane & 3)) * BPITCH2 + wn * 32 + j * 8 + (lane >> 2)];
+      for (int j = 0; j < NJ; ++j) {
+        const double2 b = bs[(kq * 4 + (lane & 3)) * BPITCH2 + wn * NJ * 8 + j * 8 + (lane >> 2)];
         br[j] = b.x; bi[j] = b.y;
       }
 #pragma unroll
-      for (int i = 0; i < 4; ++i)
+      for (int i = 0; i < MI; ++i)
 #pragma unroll
-        for (int j = 0; j < 4; ++j) {
+        for (int j = 0; j < NJ; ++j) {
           dmma(cr[i][j][0], cr[i][j][1], ar[i], br[j]);
           dmma(ci[i][j][0], ci[i][j][1], ar[i], bi[j]);
         }
 #pragma unroll
-      for (int i = 0; i < 4; ++i)
+      for (int i = 0; i < MI; ++i)
 #pragma unroll
-        for (int j = 0; j < 4; ++j) {
+        for (int j = 0; j < NJ; ++j) {
           dmma(cr[i][j][0], cr[i][j][1], an[i], bi[j]);
           dmma(ci[i][j][0], ci[i][j][1], ai[i], br[j]);
         }
@@ -365,11 +372,11 @@ __global__ void __launch_bounds__(NT, 2)
     slot_c = (slot_c + 1 == ST2) ? 0 : slot_c + 1;
     if (++kt_c == S.KTOT) {  // tile done: write back (next tile's loads already in flight)
 #pragma unroll
-      for (int i = 0; i < 4; ++i) {
-        const int m = S.m0 + wm * 32 + i * 8 + (lane >> 2);
+      for (int i = 0; i < MI; ++i) {
+        const int m = S.m0 + wm * MI * 8 + i * 8 + (lane >> 2);
 #pragma unroll
-        for (int j = 0; j < 4; ++j) {
-          const int n = S.n0 + wn * 32 + j * 8 + (lane & 3) * 2;
+        for (int j = 0; j < NJ; ++j) {
+          const int n = S.n0 + wn * NJ * 8 + j * 8 + (lane & 3) * 2;
           if (m < S.Mi) {
             double2 *cp = S.C + (long long)m * S.sCmi + (long long)n * S.sCni;
             if (n < S.Ni) cp[0] = make_double2(cr[i][j][0], ci[i][j][0]);
@@ -380,7 +387,7 @@ __global__ void __launch_bounds__(NT, 2)
       }
       kt_c = 0;
       if (++tile_c >= t_end) break;
-      decode_tile(descs, n_desc, task_c, tile_c, tid, nullptr, &S);
+      decode_tile<NTH, LPT>(descs, n_desc, task_c, tile_c, tid, (LoadCur<LPT> *)nullptr, &S);
     }
   }
   cp_async_wait<0>();
@@ -843,15 +850,17 @@ cudaError_t launch_ws(const GemmDesc *d_descs, int n, long long total, int sms, 
 
 cudaError_t launch_gemm_group(const GemmDesc *d_descs, int n, long long total_tiles, int cls, cudaStream_t st) {
   static bool attr_set = false;  // per process; the attribute is per-function, all devices
-  static int variant = -1;       // MICCO_GEMM = 1 (per-tile), 2 (persistent cp.async), 3 (default: ws)
+  static int variant = -1;  // MICCO_GEMM = 1 per-tile, 2 persistent (default), 3 warp-specialized, 5 8-warp
   if (variant < 0) {
     const char *e = getenv("MICCO_GEMM");
-    variant = (e && (e[0] == '1' || e[0] == '2')) ? e[0] - '0' : 3;
+    variant = (e && e[0] >= '1' && e[0] <= '5' && e[0] != '4') ? e[0] - '0' : 2;
   }
   if (!attr_set) {
     cudaError_t e = cudaFuncSetAttribute(zgemm_dmma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, GEMM_SMEM);
     if (e != cudaSuccess) return e;
-    e = cudaFuncSetAttribute(zgemm_dmma_persistent, cudaFuncAttributeMaxDynamicSharedMemorySize, GEMM2_SMEM);
+    e = cudaFuncSetAttribute(zgemm_dmma_persistent<2, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, GEMM2_SMEM);
+    if (e != cudaSuccess) return e;
+    e = cudaFuncSetAttribute(zgemm_dmma_persistent<2, 4>, cudaFuncAttributeMaxDynamicSharedMemorySize, GEMM2_SMEM);
     if (e != cudaSuccess) return e;
     attr_set = true;
   }
@@ -864,10 +873,13 @@ cudaError_t launch_gemm_group(const GemmDesc *d_descs, int n, long long total_ti
     zgemm_dmma_kernel<<<(unsigned)grid, NT, GEMM_SMEM, st>>>(d_descs, n, total_tiles);
     return cudaGetLastError();
   }
-  if (variant == 2) {
-    long long grid = 2LL * sms;  // 2 resident CTAs per SM (255 registers, 112 KB smem each)
+  if (variant == 2 || variant == 5) {
+    long long grid = 2LL * sms;  // 2 resident CTAs per SM (112 KB smem each)
     if (grid > total_tiles) grid = total_tiles;
-    zgemm_dmma_persistent<<<(unsigned)grid, NT, GEMM2_SMEM, st>>>(d_descs, n, total_tiles);
+    if (variant == 2)
+      zgemm_dmma_persistent<2, 2><<<(unsigned)grid, 128, GEMM2_SMEM, st>>>(d_descs, n, total_tiles);
+    else
+      zgemm_dmma_persistent<2, 4><<<(unsigned)grid, 256, GEMM2_SMEM, st>>>(d_descs, n, total_tiles);
     return cudaGetLastError();
   }
   switch (cls) {
