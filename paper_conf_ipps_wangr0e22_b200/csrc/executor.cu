@@ -95,6 +95,8 @@ micco_status nccl_unique_id(uint8_t out[128]) {
 namespace {
 
 constexpr int kRingSlots = 64;
+constexpr int kLookahead = 6;                    // chunks the H2D prefetch may run ahead
+constexpr int64_t kPrefetchBytes = 8LL << 30;    // and at most this many bytes
 constexpr size_t kSlotBytes = 256 * 1024;
 
 struct EventPool {
@@ -140,6 +142,9 @@ struct LGpu {
   cudaStream_t st = nullptr;   // compute stream: kernels, P2P, spills, frees
   cudaStream_t cst = nullptr;  // copy stream: H2D prefetch (async, overlaps the kernels)
   std::vector<cudaEvent_t> flush_ev;  // compute-stream event after each flushed chunk
+  std::vector<int64_t> chunk_fetch;   // bytes fetched for each flushed chunk
+  std::vector<int64_t> fetch_bytes_since;
+  int64_t pending_fetch = 0;          // bytes fetched for the chunk being built
   std::vector<double2 *> ptr;                                  // tensor → replica
   std::unordered_map<int32_t, std::vector<cudaEvent_t>> readers;  // peer reads to wait for before free
   std::vector<GemmDesc> gemm;
@@ -422,9 +427,11 @@ struct Executor::Impl {
       d.sBko = L.sBko; d.sBki = L.sBki; d.sBno = L.sBno; d.sBni = L.sBni;
       d.sCmo = L.sCmo; d.sCmi = L.sCmi; d.sCno = L.sCno; d.sCni = L.sCni;
       d.Lt = c.Lt;
-      d.tilesM = (L.Mi + kGemmBM - 1) / kGemmBM;
-      d.tilesN = (L.Ni + kGemmBN - 1) / kGemmBN;
       d.cls = gemm_class(L);
+      int tbm, tbn;
+      gemm_tile_shape(d.cls, &tbm, &tbn);
+      d.tilesM = (L.Mi + tbm - 1) / tbm;
+      d.tilesN = (L.Ni + tbn - 1) / tbn;
       if (fd >= 0) {  // final dot in the epilogue: C is never materialised
         const TaskRec &dk = c.tasks[fd];
         const int32_t X = tk.out, Y = dk.a == X ? dk.b : dk.a;
@@ -490,7 +497,23 @@ struct Executor::Impl {
         LGpu &l = g[op.gpu];
         if (!l.local) return;
         CK(cudaSetDevice(l.dev));
-        if (l.flush_ev.size() >= 2) CK(cudaStreamWaitEvent(l.cst, l.flush_ev[l.flush_ev.size() - 2], 0));
+        // look-ahead: the copy for stage s may run while stages s-1 .. s-kLookahead compute;
+        // bounded by bytes so the pool stays within the budget's slack (0.08 × free + 2 GiB)
+        {
+          const int64_t nb = bytes_of(op.id);
+          l.fetch_bytes_since.push_back(nb);
+          size_t nf = l.flush_ev.size();
+          int64_t ahead = 0;
+          int depth = 0;
+          // walk back over flushed chunks while the prefetch window stays small
+          while (depth < kLookahead && depth < (int)nf) {
+            ahead += l.chunk_fetch[nf - 1 - depth];
+            if (ahead > kPrefetchBytes) break;
+            ++depth;
+          }
+          if ((int)nf > depth) CK(cudaStreamWaitEvent(l.cst, l.flush_ev[nf - 1 - depth], 0));
+          l.pending_fetch += nb;
+        }
         auto it = spill_ev.find(op.id);  // a spilled intermediate: wait for its D2H
         if (it != spill_ev.end() && c.tensors[op.id].node < 0) CK(cudaStreamWaitEvent(l.cst, it->second.second, 0));
         void *p = nullptr;
@@ -574,6 +597,8 @@ struct Executor::Impl {
         if (!l.local) return;
         flush(l);
         l.flush_ev.push_back(record(op.gpu));
+        l.chunk_fetch.push_back(l.pending_fetch);
+        l.pending_fetch = 0;
         return;
       }
     }
@@ -588,7 +613,12 @@ struct Executor::Impl {
       if (l.local && l.ptr.size() < c.tensors.size()) l.ptr.resize(c.tensors.size(), nullptr);
     launches = 0;
     timed.clear();
-    for (auto &l : g) l.flush_ev.clear();
+    for (auto &l : g) {
+      l.flush_ev.clear();
+      l.chunk_fetch.clear();
+      l.fetch_bytes_since.clear();
+      l.pending_fetch = 0;
+    }
     for (auto &d : devs) { d.sync_events.reset(); d.timing_events.reset(); }
 
     PlanInput in;
@@ -599,7 +629,8 @@ struct Executor::Impl {
     in.keep_inputs = c.opt.keep_inputs_resident != 0;
     {
       const char *gv = getenv("MICCO_GEMM"), *nf = getenv("MICCO_NO_FUSE");
-      in.fuse = gv && gv[0] == '3' && !(nf && nf[0] == '1');  // the fused epilogue exists in v3 only
+      in.fuse = gemm_variant() == 3 && !(nf && nf[0] == '1');  // the fused epilogue exists in v3 only
+      (void)gv;
     }
     in.peer_gbs = (ndev > 1 && !dist()) || dist() ? 700 : 2500;
     in.host_gbs = 55;

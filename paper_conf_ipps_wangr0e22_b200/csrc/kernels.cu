@@ -176,6 +176,146 @@ __global__ void __launch_bounds__(NT, 2)
   }
 }
 
+// ---------------------------------------------------------------- small-tile GEMM (v6)
+//
+// Latency hidden by warp parallelism instead of ILP: the configuration cuBLAS picks for
+// ZGEMM on this part (ncu of cuBLAS: cutlass_80_tensorop_z884gemm_32x32_16x4, 128 threads,
+// 92 registers, 3 CTAs/SM → DMMA pipe 99.5% active; profiles/ncu_cublas_r01.txt).  CTA tile
+// TBM×TBN complex, 4 warps of (TBM/2)×(TBN/2), BK 16, TST-stage cp.async ring, one tile
+// per CTA (many resident CTAs per SM overlap each other's prologue/epilogue).
+template <int TBM, int TBN, int TST>
+struct SmallCfg {
+  static constexpr int BKs = 16;
+  static constexpr int AP = BKs + 4;   // [m][k] rows: 320 B ≡ 64 (mod 128)
+  static constexpr int BP = TBN + 2;   // [k][n] rows: (TBN+2)·16 B; TBN = 32 → 544 ≡ 32 (mod 128)
+  static constexpr int AE = TBM * AP, BE = BKs * BP;
+  static constexpr int SMEM = TST * (AE + BE) * 16;
+  static constexpr int MI = TBM / 2 / 8, NJ = TBN / 2 / 8;  // 8x8 blocks per warp
+};
+
+template <int TBM, int TBN, int TST, int MINB>
+__global__ void __launch_bounds__(128, MINB)
+    zgemm_small(const GemmDesc *__restrict__ descs, int n_desc, long long total) {
+  using Cfg = SmallCfg<TBM, TBN, TST>;
+  constexpr int BKs = Cfg::BKs, AP = Cfg::AP, BP = Cfg::BP, MI = Cfg::MI, NJ = Cfg::NJ;
+  extern __shared__ __align__(128) double2 smem[];
+  double2 *As = smem;
+  double2 *Bs = smem + TST * Cfg::AE;
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int wm = warp >> 1, wn = warp & 1;
+  const long long tile = blockIdx.x;
+  if (tile >= total) return;
+  int lo = 0, hi = n_desc - 1;
+  while (lo < hi) {
+    int mid = (lo + hi + 1) >> 1;
+    if (descs[mid].tile_begin <= tile) lo = mid; else hi = mid - 1;
+  }
+  const GemmDesc &d = descs[lo];
+  long long lt = tile - d.tile_begin;
+  const int tilesN = d.tilesN, tilesM = d.tilesM;
+  const int tn = (int)(lt % tilesN); lt /= tilesN;
+  const int tm = (int)(lt % tilesM); lt /= tilesM;
+  const int no = (int)(lt % d.No); lt /= d.No;
+  const int mo = (int)(lt % d.Mo);
+  const long long t = lt / d.Mo;
+  const int m0 = tm * TBM, n0 = tn * TBN;
+  const int Mi = d.Mi, Ni = d.Ni, Ki = d.Ki;
+  const int sAmi = (int)d.sAmi, sAki = (int)d.sAki, sBki = (int)d.sBki, sBni = (int)d.sBni;
+  const double2 *Ab = d.A + t * d.sAt + mo * d.sAmo + (long long)m0 * sAmi;
+  const double2 *Bb = d.B + t * d.sBt + no * d.sBno + (long long)n0 * sBni;
+  const bool akf = sAki == 1, bnf = sBni == 1;
+  const int KT = (Ki + BKs - 1) / BKs, KTOT = d.Ko * KT;
+  constexpr int AL = TBM * BKs / 128, BL = TBN * BKs / 128;  // copies per thread per stage
+
+  auto load = [&](int slot, int kt) {
+    const int ko = kt / KT;
+    const int kb = (kt - ko * KT) * BKs;
+    const double2 *Ak = Ab + ko * d.sAko + (long long)kb * sAki;
+    const double2 *Bk = Bb + ko * d.sBko + (long long)kb * sBki;
+    double2 *as = As + slot * Cfg::AE;
+    double2 *bs = Bs + slot * Cfg::BE;
+#pragma unroll
+    for (int j = 0; j < AL; ++j) {
+      const int e = tid + 128 * j;
+      int m, k;
+      if (akf) { k = e & (BKs - 1); m = e / BKs; } else { m = e % TBM; k = e / TBM; }
+      const bool v = (m0 + m < Mi) && (kb + k < Ki);
+      cp_async16(as + m * AP + k, v ? Ak + m * sAmi + k * sAki : d.A, v);
+    }
+#pragma unroll
+    for (int j = 0; j < BL; ++j) {
+      const int e = tid + 128 * j;
+      int n, k;
+      if (bnf) { n = e % TBN; k = e / TBN; } else { k = e & (BKs - 1); n = e / BKs; }
+      const bool v = (n0 + n < Ni) && (kb + k < Ki);
+      cp_async16(bs + k * BP + n, v ? Bk + k * sBki + n * sBni : d.B, v);
+    }
+  };
+
+  double cr[MI][NJ][2], ci[MI][NJ][2];
+#pragma unroll
+  for (int i = 0; i < MI; ++i)
+#pragma unroll
+    for (int j = 0; j < NJ; ++j) { cr[i][j][0] = cr[i][j][1] = ci[i][j][0] = ci[i][j][1] = 0.0; }
+#pragma unroll
+  for (int s = 0; s < TST - 1; ++s) {
+    if (s < KTOT) load(s, s);
+    cp_async_commit();
+  }
+  for (int kt = 0; kt < KTOT; ++kt) {
+    cp_async_wait<TST - 2>();
+    __syncthreads();
+    const int nk = kt + TST - 1;
+    if (nk < KTOT) load(nk % TST, nk);
+    cp_async_commit();
+    const double2 *as = As + (kt % TST) * Cfg::AE;
+    const double2 *bs = Bs + (kt % TST) * Cfg::BE;
+#pragma unroll
+    for (int kq = 0; kq < BKs / 4; ++kq) {
+      double ar[MI], ai[MI], br[NJ], bi[NJ];
+#pragma unroll
+      for (int i = 0; i < MI; ++i) {
+        const double2 a = as[(wm * MI * 8 + i * 8 + (lane >> 2)) * AP + kq * 4 + (lane & 3)];
+        ar[i] = a.x; ai[i] = a.y;
+      }
+#pragma unroll
+      for (int j = 0; j < NJ; ++j) {
+        const double2 b = bs[(kq * 4 + (lane & 3)) * BP + wn * NJ * 8 + j * 8 + (lane >> 2)];
+        br[j] = b.x; bi[j] = b.y;
+      }
+#pragma unroll
+      for (int i = 0; i < MI; ++i)
+#pragma unroll
+        for (int j = 0; j < NJ; ++j) {
+          dmma(cr[i][j][0], cr[i][j][1], ar[i], br[j]);
+          dmma(ci[i][j][0], ci[i][j][1], ar[i], bi[j]);
+        }
+#pragma unroll
+      for (int i = 0; i < MI; ++i)
+#pragma unroll
+        for (int j = 0; j < NJ; ++j) {
+          dmma(cr[i][j][0], cr[i][j][1], dneg(ai[i]), bi[j]);
+          dmma(ci[i][j][0], ci[i][j][1], ai[i], br[j]);
+        }
+    }
+  }
+  cp_async_wait<0>();
+  double2 *C = d.C + t * d.sCt + mo * d.sCmo + no * d.sCno;
+  const long long sCmi = d.sCmi, sCni = d.sCni;
+#pragma unroll
+  for (int i = 0; i < MI; ++i) {
+    const int m = m0 + wm * MI * 8 + i * 8 + (lane >> 2);
+    if (m >= Mi) continue;
+#pragma unroll
+    for (int j = 0; j < NJ; ++j) {
+      const int n = n0 + wn * NJ * 8 + j * 8 + (lane & 3) * 2;
+      double2 *cp = C + (long long)m * sCmi + (long long)n * sCni;
+      if (n < Ni) cp[0] = make_double2(cr[i][j][0], ci[i][j][0]);
+      if (n + 1 < Ni) cp[sCni] = make_double2(cr[i][j][1], ci[i][j][1]);
+    }
+  }
+}
+
 // ---------------------------------------------------------------- persistent GEMM (v2)
 //
 // Same math and warp tiling as zgemm_dmma_kernel, restructured to remove the per-tile
@@ -848,13 +988,29 @@ cudaError_t launch_ws(const GemmDesc *d_descs, int n, long long total, int sms, 
 }
 }  // namespace
 
-cudaError_t launch_gemm_group(const GemmDesc *d_descs, int n, long long total_tiles, int cls, cudaStream_t st) {
-  static bool attr_set = false;  // per process; the attribute is per-function, all devices
-  static int variant = -1;  // MICCO_GEMM = 1 per-tile, 2 persistent (default), 3 warp-specialized, 5 8-warp
+int gemm_variant() {
+  // MICCO_GEMM = 1 per-tile 64×64, 2 persistent 64×64, 3 warp-specialized, 5 8-warp persistent,
+  // 6 small 32×32 (4 stages, 3 CTAs/SM), 7 64×32, 8 32×32 (3 stages, 4 CTAs/SM)
+  static int variant = -1;
   if (variant < 0) {
     const char *e = getenv("MICCO_GEMM");
-    variant = (e && e[0] >= '1' && e[0] <= '5' && e[0] != '4') ? e[0] - '0' : 2;
+    variant = (e && e[0] >= '1' && e[0] <= '8' && e[0] != '4') ? e[0] - '0' : 2;
   }
+  return variant;
+}
+
+void gemm_tile_shape(int cls, int *bm, int *bn) {
+  const int v = gemm_variant();
+  *bm = 64;
+  *bn = 64;
+  if (cls == 4) return;  // gather kernel (v1)
+  if (v == 6 || v == 8) { *bm = 32; *bn = 32; }
+  if (v == 7) { *bm = 64; *bn = 32; }
+}
+
+cudaError_t launch_gemm_group(const GemmDesc *d_descs, int n, long long total_tiles, int cls, cudaStream_t st) {
+  static bool attr_set = false;  // per process; the attribute is per-function, all devices
+  const int variant = gemm_variant();
   if (!attr_set) {
     cudaError_t e = cudaFuncSetAttribute(zgemm_dmma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, GEMM_SMEM);
     if (e != cudaSuccess) return e;
@@ -871,6 +1027,27 @@ cudaError_t launch_gemm_group(const GemmDesc *d_descs, int n, long long total_ti
   if (variant == 1 || cls == 4) {
     long long grid = total_tiles < (1LL << 30) ? total_tiles : (1LL << 30);
     zgemm_dmma_kernel<<<(unsigned)grid, NT, GEMM_SMEM, st>>>(d_descs, n, total_tiles);
+    return cudaGetLastError();
+  }
+  if (variant == 6 || variant == 7 || variant == 8) {
+    // tile sizes must match the host's tilesM/tilesN (kGemmBM/BN for the other variants)
+    long long grid = total_tiles;
+    if (variant == 6) {
+      using C6 = SmallCfg<32, 32, 4>;
+      static bool a6 = false;
+      if (!a6) { cudaFuncSetAttribute(zgemm_small<32, 32, 4, 3>, cudaFuncAttributeMaxDynamicSharedMemorySize, C6::SMEM); a6 = true; }
+      zgemm_small<32, 32, 4, 3><<<(unsigned)grid, 128, C6::SMEM, st>>>(d_descs, n, total_tiles);
+    } else if (variant == 7) {
+      using C7 = SmallCfg<64, 32, 4>;
+      static bool a7 = false;
+      if (!a7) { cudaFuncSetAttribute(zgemm_small<64, 32, 4, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, C7::SMEM); a7 = true; }
+      zgemm_small<64, 32, 4, 2><<<(unsigned)grid, 128, C7::SMEM, st>>>(d_descs, n, total_tiles);
+    } else {
+      using C8 = SmallCfg<32, 32, 3>;
+      static bool a8 = false;
+      if (!a8) { cudaFuncSetAttribute(zgemm_small<32, 32, 3, 4>, cudaFuncAttributeMaxDynamicSharedMemorySize, C8::SMEM); a8 = true; }
+      zgemm_small<32, 32, 3, 4><<<(unsigned)grid, 128, C8::SMEM, st>>>(d_descs, n, total_tiles);
+    }
     return cudaGetLastError();
   }
   if (variant == 2 || variant == 5) {

@@ -61,6 +61,11 @@ constexpr int kGemmBM = 64, kGemmBN = 64, kGemmBK = 8, kGemmStages = 4, kGemmThr
 // inner index for both operands (warp-specialized kernel), 4 = generic gather kernel.
 constexpr int kGemmClasses = 5;
 
+// The GEMM kernel variant in use (env MICCO_GEMM, see kernels.cu) and its CTA tile (complex
+// elements) for a layout class; tilesM/tilesN of a descriptor must use this shape.
+int gemm_variant();
+void gemm_tile_shape(int cls, int *bm, int *bn);
+
 // Grouped launches: descs in device memory (all of one layout class); grid covers the tiles.
 cudaError_t launch_gemm_group(const GemmDesc *d_descs, int n, long long total_tiles, int cls, cudaStream_t st);
 cudaError_t launch_dot_group(const DotDesc *d_descs, int n, long long total_ctas, cudaStream_t st);
