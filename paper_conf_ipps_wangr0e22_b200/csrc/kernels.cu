@@ -550,7 +550,8 @@ __global__ void __launch_bounds__(NWM * NWN * 32, 2)
 // inner index use zgemm_dmma_kernel.
 
 constexpr int NCW = 4;                    // consumer warps
-constexpr int NT3 = (NCW + 1) * 32;       // + 1 producer warp
+constexpr int NPW = 4;                    // producer warps (outstanding cp.async spread over 128 lanes)
+constexpr int NT3 = (NCW + NPW) * 32;
 constexpr int PITCH_MK = BK2 + 4;         // [m][k] / [n][k]: 320 B rows
 constexpr int PITCH_KM = BM + 2;          // [k][m] / [k][n]: 1056 B rows
 
@@ -640,15 +641,15 @@ __global__ void __launch_bounds__(NT3, 1)
   }
   if (tid == 0) {
     for (int s = 0; s < ST3; ++s) {
-      mbar_init(smem_u32(&bars[s]), 32);
+      mbar_init(smem_u32(&bars[s]), 32 * NPW);
       mbar_init(smem_u32(&bars[ST3 + s]), NCW);
     }
     asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
   }
   __syncthreads();
 
-  if (warp == 0) {
-    // ------------------------------------------------------------ producer warp
+  if (warp < NPW) {
+    // ------------------------------------------------------------ producer warps
     // Warp 0 on purpose: the SMSP arbiter favours the highest warp id, so the DMMA warp that
     // shares this SMSP (warp 4) wins every issue slot it can use and the producer fills the
     // cycles between its DMMAs (with the producer as warp 4 the CTA ran at the pace of the
@@ -679,8 +680,8 @@ __global__ void __launch_bounds__(NT3, 1)
         double2 *as = smem + slot * Cfg::STAGE;
         double2 *bs = as + Cfg::A_ELEMS;
 #pragma unroll 4
-        for (int j = 0; j < (BM * BK2) / 32; ++j) {
-          const int e = lane + 32 * j;
+        for (int j = 0; j < (BM * BK2) / (32 * NPW); ++j) {
+          const int e = tid + 32 * NPW * j;
           int m, k;
           if (A_MK) { k = e & (BK2 - 1); m = e / BK2; } else { m = e & (BM - 1); k = e / BM; }
           const bool v = m < mv && k < kv;
@@ -688,8 +689,8 @@ __global__ void __launch_bounds__(NT3, 1)
           cp_async16(A_MK ? as + m * PITCH_MK + k : as + k * PITCH_KM + m, src, v);
         }
 #pragma unroll 4
-        for (int j = 0; j < (BN * BK2) / 32; ++j) {
-          const int e = lane + 32 * j;
+        for (int j = 0; j < (BN * BK2) / (32 * NPW); ++j) {
+          const int e = tid + 32 * NPW * j;
           int n, k;
           if (B_KN) { n = e & (BN - 1); k = e / BN; } else { k = e & (BK2 - 1); n = e / BK2; }
           const bool v = n < nv && k < kv;
@@ -707,7 +708,7 @@ __global__ void __launch_bounds__(NT3, 1)
   // One consumer warp per SMSP: it must issue a DMMA every 16 cycles, so its shared-memory
   // fragment loads for k-quad q+1 are issued before the DMMAs of q (double-buffered
   // fragments), and the next stage is awaited one k-quad early.
-  const int cw = warp - 1;  // consumer index 0..3
+  const int cw = warp - NPW;  // consumer index 0..3
   const int wm = cw >> 1, wn = cw & 1;
   double cr[4][4][2], ci[4][4][2];
 #pragma unroll
