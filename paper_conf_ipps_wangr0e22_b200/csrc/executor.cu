@@ -255,6 +255,11 @@ struct Executor::Impl {
         CK(cudaDeviceGetDefaultMemPool(&pool, l.dev));
         uint64_t thr = UINT64_MAX;
         CK(cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr));
+        // never let an allocation on one stream wait for a free on another: the H2D prefetch
+        // on the copy stream must not be serialised behind the compute stream (the driver
+        // would otherwise insert a dependency to reuse a block freed by the compute stream)
+        int no = 0;
+        CK(cudaMemPoolSetAttribute(pool, cudaMemPoolReuseAllowInternalDependencies, &no));
         for (int p = 0; p < ndev; ++p) {  // NVLink peer access for P2P replicas
           if (p == l.dev) continue;
           int can = 0;
