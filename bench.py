@@ -231,6 +231,8 @@ def main():
         e2e_ms.append(max_over_ranks(ms))
         e2e_h2d.append(st["bytes_h2d"])
         e2e_copy.append(st["copy_ms"])
+        e2e_enq = st["enqueue_ms"]
+        e2e_pinned = st["host_pinned"]
         e2e_d2h.append(wl.Lt * 16)
     # ---- warm: inputs resident in HBM (left cached by the cold run)
     ctx.execute(world)
@@ -303,7 +305,8 @@ def main():
         "e2e": ({"value": G / (statistics.mean(e2e_ms) / 1e3), "unit": "graphs/s",
                  "h2d_bytes_per_step": int(statistics.mean(e2e_h2d)), "d2h_bytes_per_step": int(e2e_d2h[0]),
                  "ms_per_step": statistics.mean(e2e_ms),
-                 "h2d_device_ms_per_step": statistics.mean(e2e_copy)} if e2e_ms else None),
+                 "h2d_device_ms_per_step": statistics.mean(e2e_copy),
+                 "host_enqueue_ms": e2e_enq, "host_pinned": e2e_pinned} if e2e_ms else None),
         "gpu_launches": launches,
         "clocks": clk,
         "sched_ms_per_step": statistics.mean(s["sched_ms"] for s in stats),

@@ -183,6 +183,9 @@ typedef struct {
   int64_t gemm_launches, dot_launches;
   double gemm_flops;           /* algorithmic flops of the GEMM-shaped tasks executed */
   double dot_bytes;            /* algorithmic bytes read by the dot/trace tasks executed */
+  double enqueue_ms;           /* host time spent replaying the plan (issuing copies/kernels) */
+  int32_t host_pinned;         /* 1 if every node tensor lives in page-locked host memory */
+  int32_t reserved0;
 } micco_stats;
 
 MICCO_API micco_status micco_get_stats(const micco_ctx *ctx, micco_stats *out);

@@ -691,7 +691,10 @@ struct Executor::Impl {
           CK(cudaStreamWaitEvent(g[i].st, e, 0));
         }
     }
+    auto tq0 = std::chrono::steady_clock::now();
     for (const PlanOp &op : plan.ops) run_op(op, st);
+    st.enqueue_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - tq0).count();
+    st.host_pinned = c.arena.pinned() ? 1 : 0;
     for (auto &l : g)
       if (l.local && (!l.gemm.empty() || !l.dot.empty())) flush(l);
     // intermediates must all be released by now; drop leftovers defensively

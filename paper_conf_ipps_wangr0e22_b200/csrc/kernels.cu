@@ -845,8 +845,10 @@ __device__ __forceinline__ void cmac(double &sr, double &si, double2 a, double2 
   si += a.x * b.y + a.y * b.x;
 }
 
+constexpr int DOT_SMEM = (DT / 32) * 32 * 17 * 16;  // one 32×17 complex slab per warp (69.6 KB)
+
 __global__ void __launch_bounds__(DT) zdot_kernel(const DotDesc *__restrict__ descs, int n_desc) {
-  __shared__ double2 As[32][33], Bs[32][33];
+  extern __shared__ __align__(16) double2 dsm[];
   __shared__ double red[2][DT / 32];
   const long long cta = blockIdx.x;
   int lo = 0, hi = n_desc - 1;
@@ -876,6 +878,7 @@ __global__ void __launch_bounds__(DT) zdot_kernel(const DotDesc *__restrict__ de
     }
   } else if (d.mode == 0) {
     const long long X = d.X, total = Ototal * X;
+#pragma unroll 4
     for (long long e = tid; e < total; e += DT) {
       const long long o = e / X, x = e - o * X;
       const long long o2 = o % O2, o01 = o / O2, o1 = o01 % O1, o0 = o01 / O1;
@@ -883,24 +886,40 @@ __global__ void __launch_bounds__(DT) zdot_kernel(const DotDesc *__restrict__ de
       const long long offB = o0 * d.sBo[0] + o1 * d.sBo[1] + o2 * d.sBo[2] + x * d.sBx;
       cmac(sr, si, A[offA], B[offB]);
     }
-  } else {  // transpose tiles: A contiguous along x, B contiguous along y
-    const int ty = tid >> 5, tx = tid & 31;
-    for (long long o = 0; o < Ototal; ++o) {
+  } else {
+    // transposed pair (A contiguous along x, B along y): every warp owns 32(x)×16(y) sub-tiles;
+    // A rows stay in registers (16 independent coalesced loads per lane), the B block goes
+    // through the warp's own padded smem slab (16 coalesced loads per lane), so no CTA-wide
+    // barrier and 32 loads in flight per lane.
+    double2 *Bs = dsm + (tid >> 5) * (32 * 17);
+    const int lane = tid & 31;
+    const int nx = (d.X + 31) / 32, ny = (d.Y + 15) / 16;
+    const long long nsub = Ototal * nx * ny;
+    for (long long sub = tid >> 5; sub < nsub; sub += DT / 32) {
+      const long long o = sub / (nx * ny);
+      const int rem = (int)(sub - o * nx * ny);
+      const int y0 = (rem / nx) * 16, x0 = (rem % nx) * 32;
       const long long o2 = o % O2, o01 = o / O2, o1 = o01 % O1, o0 = o01 / O1;
       const double2 *Ao = A + o0 * d.sAo[0] + o1 * d.sAo[1] + o2 * d.sAo[2];
       const double2 *Bo = B + o0 * d.sBo[0] + o1 * d.sBo[1] + o2 * d.sBo[2];
-      for (int y0 = 0; y0 < d.Y; y0 += 32)
-        for (int x0 = 0; x0 < d.X; x0 += 32) {
-          for (int r = ty; r < 32; r += DT / 32) {
-            const int y = y0 + r, x = x0 + tx;
-            As[r][tx] = (y < d.Y && x < d.X) ? Ao[(long long)y * d.sAy + (long long)x * d.sAx] : make_double2(0, 0);
-            const int xb = x0 + r, yb = y0 + tx;
-            Bs[r][tx] = (xb < d.X && yb < d.Y) ? Bo[(long long)xb * d.sBx + (long long)yb * d.sBy] : make_double2(0, 0);
-          }
-          __syncthreads();
-          for (int r = ty; r < 32; r += DT / 32) cmac(sr, si, As[r][tx], Bs[tx][r]);
-          __syncthreads();
-        }
+      double2 a[16];
+      const int x = x0 + lane;
+#pragma unroll
+      for (int r = 0; r < 16; ++r) {
+        const int y = y0 + r;
+        a[r] = (y < d.Y && x < d.X) ? Ao[(long long)y * d.sAy + (long long)x * d.sAx] : make_double2(0.0, 0.0);
+      }
+      __syncwarp();
+#pragma unroll
+      for (int rr = 0; rr < 16; ++rr) {
+        const int xl = 2 * rr + (lane >> 4), yl = lane & 15;
+        const int xb = x0 + xl, yb = y0 + yl;
+        Bs[xl * 17 + yl] = (xb < d.X && yb < d.Y) ? Bo[(long long)xb * d.sBx + (long long)yb * d.sBy]
+                                                  : make_double2(0.0, 0.0);
+      }
+      __syncwarp();
+#pragma unroll
+      for (int r = 0; r < 16; ++r) cmac(sr, si, a[r], Bs[lane * 17 + r]);
     }
   }
   // deterministic block reduction: xor butterfly, then warps in order
@@ -1070,7 +1089,13 @@ cudaError_t launch_gemm_group(const GemmDesc *d_descs, int n, long long total_ti
 
 cudaError_t launch_dot_group(const DotDesc *d_descs, int n, long long total_ctas, cudaStream_t st) {
   if (total_ctas <= 0) return cudaSuccess;
-  zdot_kernel<<<(unsigned)total_ctas, DT, 0, st>>>(d_descs, n);
+  static bool attr = false;
+  if (!attr) {
+    cudaError_t e = cudaFuncSetAttribute(zdot_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, DOT_SMEM);
+    if (e != cudaSuccess) return e;
+    attr = true;
+  }
+  zdot_kernel<<<(unsigned)total_ctas, DT, DOT_SMEM, st>>>(d_descs, n);
   return cudaGetLastError();
 }
 
