@@ -7,8 +7,8 @@
 //    replicas held by another GPU, D2H spills of sole copies under memory pressure
 //    (allocation and CPU↔GPU / GPU↔GPU movement are the memory
 //    operations the scheduler trades against load balance);
-//  * the tasks of one stage and GPU are batched into one grouped GEMM launch and one grouped
-//    dot launch (descriptors staged through a pinned ring);
+//  * the tasks of one stage and GPU are batched into grouped GEMM launches (one per operand
+//    layout class) and one grouped dot launch; descriptors are kernel parameters;
 //  * rank-0 results land in a per-device scalar table [slot][t]; devices are combined by an
 //    exact sum (each slot is nonzero on one device only): NCCL all-reduce in multi-process
 //    mode, peer copies otherwise; then C(t) = Σ_g c_g Π_comp s_comp(t) on device 0.
@@ -23,6 +23,7 @@
 #include <cstdlib>
 #include <cstring>
 #include <string>
+#include <type_traits>
 #include <unordered_map>
 
 #include "executor.h"
@@ -94,10 +95,8 @@ micco_status nccl_unique_id(uint8_t out[128]) {
 
 namespace {
 
-constexpr int kRingSlots = 64;
 constexpr int kLookahead = 6;                    // chunks the H2D prefetch may run ahead
 constexpr int64_t kPrefetchBytes = 8LL << 30;    // and at most this many bytes
-constexpr size_t kSlotBytes = 256 * 1024;
 
 struct EventPool {
   int dev = -1;
@@ -151,10 +150,6 @@ struct LGpu {
   std::vector<DotDesc> dot;
   std::vector<double2 *> part_allocs;  // fused-dot partials of the pending batch
   long long gemm_tiles = 0, dot_ctas = 0;
-  char *ring_h = nullptr, *ring_d = nullptr;
-  cudaEvent_t ring_ev[kRingSlots] = {};
-  bool ring_used[kRingSlots] = {};
-  int ring_next = 0;
 };
 
 }  // namespace
@@ -175,6 +170,8 @@ struct Executor::Impl {
   int budget_cache_n = 0;
   std::vector<std::pair<int32_t, uint64_t>> cached_nodes;
   std::vector<int32_t> fused_dot;  // of the plan being replayed
+  std::unique_ptr<GemmBatch> gemm_batch{new GemmBatch};  // kernel-parameter staging
+  std::unique_ptr<DotBatch> dot_batch{new DotBatch};
   int32_t chosen_bd[3] = {0, 0, 0};
   int chosen_bd_n = 0;
   // results on device 0
@@ -217,10 +214,6 @@ struct Executor::Impl {
     if (l.cst) cudaStreamSynchronize(l.cst);
     l.readers.clear();
     if (destroy_stream) {
-      for (int i = 0; i < kRingSlots; ++i)
-        if (l.ring_ev[i]) cudaEventDestroy(l.ring_ev[i]);
-      if (l.ring_h) cudaFreeHost(l.ring_h);
-      if (l.ring_d) cudaFree(l.ring_d);
       cudaStreamDestroy(l.st);
       cudaStreamDestroy(l.cst);
       l.st = nullptr;
@@ -274,9 +267,6 @@ struct Executor::Impl {
       }
       CK(cudaStreamCreateWithFlags(&l.st, cudaStreamNonBlocking));
       CK(cudaStreamCreateWithFlags(&l.cst, cudaStreamNonBlocking));
-      CK(cudaHostAlloc((void **)&l.ring_h, kRingSlots * kSlotBytes, cudaHostAllocPortable));
-      CK(cudaMalloc((void **)&l.ring_d, kRingSlots * kSlotBytes));
-      for (int s = 0; s < kRingSlots; ++s) CK(cudaEventCreateWithFlags(&l.ring_ev[s], cudaEventDisableTiming));
     }
     if (dist()) {
       if (!c.have_nccl_id) fail(MICCO_ERR_STATE, "multi-process mode needs micco_set_nccl_id before execute");
@@ -344,33 +334,18 @@ struct Executor::Impl {
     return it->second;
   }
 
-  char *ring_slot(LGpu &l, size_t bytes, int &slot) {
-    if (bytes > kSlotBytes) fail(MICCO_ERR_STATE, "descriptor batch too large");
-    slot = l.ring_next;
-    l.ring_next = (l.ring_next + 1) % kRingSlots;
-    if (l.ring_used[slot]) CK(cudaEventSynchronize(l.ring_ev[slot]));
-    l.ring_used[slot] = true;
-    return l.ring_h + (size_t)slot * kSlotBytes;
-  }
-
-  template <typename D, typename Launch>
-  void launch_batch(LGpu &l, std::vector<D> &v, int kind, int cls, Launch &&prefix) {
+  template <typename D, typename Batch, typename Prefix>
+  void launch_batch(LGpu &l, std::vector<D> &v, int kind, int cls, Batch &b, int cap, Prefix &&prefix) {
     if (v.empty()) return;
-    const size_t per = kSlotBytes / sizeof(D);
-    for (size_t i0 = 0; i0 < v.size(); i0 += per) {
-      size_t cnt = std::min(per, v.size() - i0);
-      int slot;
-      char *h = ring_slot(l, cnt * sizeof(D), slot);
-      std::memcpy(h, &v[i0], cnt * sizeof(D));
-      D *hd = (D *)h;
-      const long long total = prefix(hd, (int)cnt);  // grid offsets in the staged copy
-      char *dptr = l.ring_d + (size_t)slot * kSlotBytes;
-      CK(cudaMemcpyAsync(dptr, h, cnt * sizeof(D), cudaMemcpyHostToDevice, l.st));
-      CK(cudaEventRecord(l.ring_ev[slot], l.st));
+    for (size_t i0 = 0; i0 < v.size(); i0 += (size_t)cap) {
+      const int cnt = (int)std::min((size_t)cap, v.size() - i0);
+      b.n = cnt;
+      std::memcpy(b.d, &v[i0], cnt * sizeof(D));
+      const long long total = prefix(b.d, cnt);  // grid offsets of this launch
       Timed tm{devs[l.dev].timing_events.get(), devs[l.dev].timing_events.get(), kind, l.dev};
       CK(cudaEventRecord(tm.a, l.st));
-      if (kind == 0) CK(launch_gemm_group((const GemmDesc *)dptr, (int)cnt, total, cls, l.st));
-      else CK(launch_dot_group((const DotDesc *)dptr, (int)cnt, total, l.st));
+      if constexpr (std::is_same<D, GemmDesc>::value) CK(launch_gemm_group(&b, total, cls, l.st));
+      else CK(launch_dot_group(&b, total, l.st));
       CK(cudaEventRecord(tm.b, l.st));
       timed.push_back(tm);
       ++launches;
@@ -385,7 +360,7 @@ struct Executor::Impl {
       for (const GemmDesc &d : l.gemm) by[d.cls].push_back(d);
       l.gemm.clear();
       for (int c = 0; c < kGemmClasses; ++c)
-        launch_batch(l, by[c], 0, c, [](GemmDesc *d, int cnt) {
+        launch_batch(l, by[c], 0, c, *gemm_batch, kGemmBatch, [](GemmDesc *d, int cnt) {
           long long acc = 0;
           for (int i = 0; i < cnt; ++i) {
             d[i].tile_begin = acc;
@@ -394,7 +369,7 @@ struct Executor::Impl {
           return acc;
         });
     }
-    launch_batch(l, l.dot, 1, 0, [](DotDesc *d, int cnt) {
+    launch_batch(l, l.dot, 1, 0, *dot_batch, kDotBatch, [](DotDesc *d, int cnt) {
       long long acc = 0;
       for (int i = 0; i < cnt; ++i) {
         d[i].cta_begin = acc;

@@ -59,8 +59,8 @@ __device__ __forceinline__ int find_desc(const D *descs, int n, long long item) 
   return lo;
 }
 
-__global__ void __launch_bounds__(NT, 2)
-    zgemm_dmma_kernel(const GemmDesc *__restrict__ descs, int n_desc, long long total) {
+__device__ __forceinline__ void zgemm_dmma_kernel_body(const GemmDesc *__restrict__ descs, int n_desc,
+                                                       long long total) {
   extern __shared__ __align__(128) double2 smem[];
   double2 *As = smem;
   double2 *Bs = smem + ST * A_STAGE;
@@ -193,9 +193,8 @@ struct SmallCfg {
   static constexpr int MI = TBM / 2 / 8, NJ = TBN / 2 / 8;  // 8x8 blocks per warp
 };
 
-template <int TBM, int TBN, int TST, int MINB>
-__global__ void __launch_bounds__(128, MINB)
-    zgemm_small(const GemmDesc *__restrict__ descs, int n_desc, long long total) {
+template <int TBM, int TBN, int TST>
+__device__ __forceinline__ void zgemm_small_body(const GemmDesc *__restrict__ descs, int n_desc, long long total) {
   using Cfg = SmallCfg<TBM, TBN, TST>;
   constexpr int BKs = Cfg::BKs, AP = Cfg::AP, BP = Cfg::BP, MI = Cfg::MI, NJ = Cfg::NJ;
   extern __shared__ __align__(128) double2 smem[];
@@ -398,8 +397,8 @@ __device__ __forceinline__ void decode_tile(const GemmDesc *__restrict__ descs, 
 // warp tiles (248-255 registers, 2 warps per SMSP); <2,4> = 256 threads with 32×16 warp
 // tiles (half the accumulators, 4 warps per SMSP for latency hiding).
 template <int NWM, int NWN>
-__global__ void __launch_bounds__(NWM * NWN * 32, 2)
-    zgemm_dmma_persistent(const GemmDesc *__restrict__ descs, int n_desc, long long total) {
+__device__ __forceinline__ void zgemm_dmma_persistent_body(const GemmDesc *__restrict__ descs, int n_desc,
+                                                           long long total) {
   constexpr int NTH = NWM * NWN * 32, LPT = (BM * BK2) / NTH;
   constexpr int MI = BM / NWM / 8, NJ = BN / NWN / 8;  // 8x8 blocks per warp
   extern __shared__ __align__(128) double2 smem[];
@@ -430,35 +429,52 @@ __global__ void __launch_bounds__(NWM * NWN * 32, 2)
   decode_tile<NTH, LPT>(descs, n_desc, task_c, tile_c, tid, (LoadCur<LPT> *)nullptr, &S);
   bool more_l = true;
 
-  auto issue_load = [&](int slot) {
+  // The loads of a stage are issued in NPART pieces interleaved with the DMMA stream of the
+  // stage being computed (one piece per k-quad), so the scheduler can slot the cp.async and
+  // address arithmetic into the DMMA pacing gaps instead of running a separate load phase.
+  constexpr int NPART = BK2 / 4;
+  const double2 *ldA = nullptr, *ldB = nullptr;
+  int ld_kb = 0;
+  auto begin_load = [&]() {
     const int ko = kt_l / L.KT;
-    const int kb = (kt_l - ko * L.KT) * BK2;
-    const double2 *Ak = L.A + ko * L.sAko + (long long)kb * L.sAki;
-    const double2 *Bk = L.B + ko * L.sBko + (long long)kb * L.sBki;
+    ld_kb = (kt_l - ko * L.KT) * BK2;
+    ldA = L.A + ko * L.sAko + (long long)ld_kb * L.sAki;
+    ldB = L.B + ko * L.sBko + (long long)ld_kb * L.sBki;
+  };
+  auto issue_part = [&](int slot, int part) {
     double2 *as = As + slot * A_STAGE2;
     double2 *bs = Bs + slot * B_STAGE2;
 #pragma unroll
-    for (int j = 0; j < LPT; ++j) {
+    for (int jj = 0; jj < LPT / NPART; ++jj) {
+      const int j = part * (LPT / NPART) + jj;
       const int e = tid + j * NTH;
       int m, k;
       if (L.akf) { k = e & (BK2 - 1); m = e / BK2; } else { m = e & (BM - 1); k = e / BM; }
-      const bool v = ((L.vA >> j) & 1u) && (kb + k < L.Ki);
-      cp_async16(as + m * APITCH2 + k, v ? Ak + L.offA[j] : L.A, v);
+      const bool v = ((L.vA >> j) & 1u) && (ld_kb + k < L.Ki);
+      cp_async16(as + m * APITCH2 + k, v ? ldA + L.offA[j] : L.A, v);
     }
 #pragma unroll
-    for (int j = 0; j < LPT; ++j) {
+    for (int jj = 0; jj < LPT / NPART; ++jj) {
+      const int j = part * (LPT / NPART) + jj;
       const int e = tid + j * NTH;
       int n, k;
       if (L.bnf) { n = e & (BN - 1); k = e / BN; } else { k = e & (BK2 - 1); n = e / BK2; }
-      const bool v = ((L.vB >> j) & 1u) && (kb + k < L.Ki);
-      cp_async16(bs + k * BPITCH2 + n, v ? Bk + L.offB[j] : L.B, v);
+      const bool v = ((L.vB >> j) & 1u) && (ld_kb + k < L.Ki);
+      cp_async16(bs + k * BPITCH2 + n, v ? ldB + L.offB[j] : L.B, v);
     }
-    // advance the load cursor (possibly into the next tile)
+  };
+  auto advance_load = [&]() {  // next k-step, possibly in the next tile
     if (++kt_l == L.KTOT) {
       kt_l = 0;
       if (++tile_l < t_end) decode_tile<NTH, LPT>(descs, n_desc, task_l, tile_l, tid, &L, nullptr);
       else more_l = false;
     }
+  };
+  auto issue_load = [&](int slot) {
+    begin_load();
+#pragma unroll
+    for (int p = 0; p < NPART; ++p) issue_part(slot, p);
+    advance_load();
   };
 
   double cr[MI][NJ][2], ci[MI][NJ][2];
@@ -476,13 +492,13 @@ __global__ void __launch_bounds__(NWM * NWN * 32, 2)
   for (;;) {
     cp_async_wait<ST2 - 2>();
     __syncthreads();
-    if (more_l) issue_load(slot_l);
-    cp_async_commit();
-    slot_l = (slot_l + 1 == ST2) ? 0 : slot_l + 1;
+    const bool ld = more_l;
+    if (ld) begin_load();
     const double2 *as = As + slot_c * A_STAGE2;
     const double2 *bs = Bs + slot_c * B_STAGE2;
 #pragma unroll
     for (int kq = 0; kq < BK2 / 4; ++kq) {
+      if (ld) issue_part(slot_l, kq);
       double ar[MI], ai[MI], an[MI], br[NJ], bi[NJ];
 #pragma unroll
       for (int i = 0; i < MI; ++i) {
@@ -509,6 +525,9 @@ __global__ void __launch_bounds__(NWM * NWN * 32, 2)
           dmma(ci[i][j][0], ci[i][j][1], ai[i], br[j]);
         }
     }
+    if (ld) advance_load();
+    cp_async_commit();
+    slot_l = (slot_l + 1 == ST2) ? 0 : slot_l + 1;
     slot_c = (slot_c + 1 == ST2) ? 0 : slot_c + 1;
     if (++kt_c == S.KTOT) {  // tile done: write back (next tile's loads already in flight)
 #pragma unroll
@@ -618,8 +637,7 @@ __device__ __forceinline__ void v3_decode(const GemmDesc *__restrict__ descs, in
 }
 
 template <bool A_MK, bool B_KN>
-__global__ void __launch_bounds__(NT3, 1)
-    zgemm_dmma_ws(const GemmDesc *__restrict__ descs, int n_desc, long long total) {
+__device__ __forceinline__ void zgemm_dmma_ws_body(const GemmDesc *__restrict__ descs, int n_desc, long long total) {
   using Cfg = V3Cfg<A_MK, B_KN>;
   constexpr int ST3 = Cfg::ST;
   extern __shared__ __align__(128) double2 smem[];
@@ -847,7 +865,7 @@ __device__ __forceinline__ void cmac(double &sr, double &si, double2 a, double2 
 
 constexpr int DOT_SMEM = (DT / 32) * 32 * 17 * 16;  // one 32×17 complex slab per warp (69.6 KB)
 
-__global__ void __launch_bounds__(DT) zdot_kernel(const DotDesc *__restrict__ descs, int n_desc) {
+__device__ __forceinline__ void zdot_body(const DotDesc *__restrict__ descs, int n_desc) {
   extern __shared__ __align__(16) double2 dsm[];
   __shared__ double red[2][DT / 32];
   const long long cta = blockIdx.x;
@@ -988,11 +1006,30 @@ __global__ void accumulate_kernel(double2 *dst, const double2 *src, long long n)
   }
 }
 
-}  // namespace
 
-namespace {
+// Kernel entry points.  Descriptors travel as __grid_constant__ kernel parameters (up to
+// 32 KB per launch on sm_100): no H2D memcpy on the compute stream, which would otherwise
+// queue behind the node prefetch copies on the copy engine and serialise compute behind H2D.
+__global__ void __launch_bounds__(NT, 2) zgemm_dmma_kernel(const __grid_constant__ GemmBatch b, long long total) {
+  zgemm_dmma_kernel_body(b.d, b.n, total);
+}
+template <int TBM, int TBN, int TST, int MINB>
+__global__ void __launch_bounds__(128, MINB) zgemm_small(const __grid_constant__ GemmBatch b, long long total) {
+  zgemm_small_body<TBM, TBN, TST>(b.d, b.n, total);
+}
+template <int NWM, int NWN>
+__global__ void __launch_bounds__(NWM * NWN * 32, 2)
+    zgemm_dmma_persistent(const __grid_constant__ GemmBatch b, long long total) {
+  zgemm_dmma_persistent_body<NWM, NWN>(b.d, b.n, total);
+}
 template <bool A_MK, bool B_KN>
-cudaError_t launch_ws(const GemmDesc *d_descs, int n, long long total, int sms, cudaStream_t st) {
+__global__ void __launch_bounds__(NT3, 1) zgemm_dmma_ws(const __grid_constant__ GemmBatch b, long long total) {
+  zgemm_dmma_ws_body<A_MK, B_KN>(b.d, b.n, total);
+}
+__global__ void __launch_bounds__(DT) zdot_kernel(const __grid_constant__ DotBatch b) { zdot_body(b.d, b.n); }
+
+template <bool A_MK, bool B_KN>
+cudaError_t launch_ws(const GemmBatch *b, long long total, int sms, cudaStream_t st) {
   using Cfg = V3Cfg<A_MK, B_KN>;
   static bool attr = false;
   if (!attr) {
@@ -1003,9 +1040,10 @@ cudaError_t launch_ws(const GemmDesc *d_descs, int n, long long total, int sms, 
   }
   long long grid = sms;  // one CTA (4 DMMA warps + 1 producer) per SM
   if (grid > total) grid = total;
-  zgemm_dmma_ws<A_MK, B_KN><<<(unsigned)grid, NT3, Cfg::SMEM, st>>>(d_descs, n, total);
+  zgemm_dmma_ws<A_MK, B_KN><<<(unsigned)grid, NT3, Cfg::SMEM, st>>>(*b, total);
   return cudaGetLastError();
 }
+
 }  // namespace
 
 int gemm_variant() {
@@ -1028,7 +1066,7 @@ void gemm_tile_shape(int cls, int *bm, int *bn) {
   if (v == 7) { *bm = 64; *bn = 32; }
 }
 
-cudaError_t launch_gemm_group(const GemmDesc *d_descs, int n, long long total_tiles, int cls, cudaStream_t st) {
+cudaError_t launch_gemm_group(const GemmBatch *b, long long total_tiles, int cls, cudaStream_t st) {
   static bool attr_set = false;  // per process; the attribute is per-function, all devices
   const int variant = gemm_variant();
   if (!attr_set) {
@@ -1046,7 +1084,7 @@ cudaError_t launch_gemm_group(const GemmDesc *d_descs, int n, long long total_ti
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   if (variant == 1 || cls == 4) {
     long long grid = total_tiles < (1LL << 30) ? total_tiles : (1LL << 30);
-    zgemm_dmma_kernel<<<(unsigned)grid, NT, GEMM_SMEM, st>>>(d_descs, n, total_tiles);
+    zgemm_dmma_kernel<<<(unsigned)grid, NT, GEMM_SMEM, st>>>(*b, total_tiles);
     return cudaGetLastError();
   }
   if (variant == 6 || variant == 7 || variant == 8) {
@@ -1056,17 +1094,17 @@ cudaError_t launch_gemm_group(const GemmDesc *d_descs, int n, long long total_ti
       using C6 = SmallCfg<32, 32, 4>;
       static bool a6 = false;
       if (!a6) { cudaFuncSetAttribute(zgemm_small<32, 32, 4, 3>, cudaFuncAttributeMaxDynamicSharedMemorySize, C6::SMEM); a6 = true; }
-      zgemm_small<32, 32, 4, 3><<<(unsigned)grid, 128, C6::SMEM, st>>>(d_descs, n, total_tiles);
+      zgemm_small<32, 32, 4, 3><<<(unsigned)grid, 128, C6::SMEM, st>>>(*b, total_tiles);
     } else if (variant == 7) {
       using C7 = SmallCfg<64, 32, 4>;
       static bool a7 = false;
       if (!a7) { cudaFuncSetAttribute(zgemm_small<64, 32, 4, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, C7::SMEM); a7 = true; }
-      zgemm_small<64, 32, 4, 2><<<(unsigned)grid, 128, C7::SMEM, st>>>(d_descs, n, total_tiles);
+      zgemm_small<64, 32, 4, 2><<<(unsigned)grid, 128, C7::SMEM, st>>>(*b, total_tiles);
     } else {
       using C8 = SmallCfg<32, 32, 3>;
       static bool a8 = false;
       if (!a8) { cudaFuncSetAttribute(zgemm_small<32, 32, 3, 4>, cudaFuncAttributeMaxDynamicSharedMemorySize, C8::SMEM); a8 = true; }
-      zgemm_small<32, 32, 3, 4><<<(unsigned)grid, 128, C8::SMEM, st>>>(d_descs, n, total_tiles);
+      zgemm_small<32, 32, 3, 4><<<(unsigned)grid, 128, C8::SMEM, st>>>(*b, total_tiles);
     }
     return cudaGetLastError();
   }
@@ -1074,20 +1112,20 @@ cudaError_t launch_gemm_group(const GemmDesc *d_descs, int n, long long total_ti
     long long grid = 2LL * sms;  // 2 resident CTAs per SM (112 KB smem each)
     if (grid > total_tiles) grid = total_tiles;
     if (variant == 2)
-      zgemm_dmma_persistent<2, 2><<<(unsigned)grid, 128, GEMM2_SMEM, st>>>(d_descs, n, total_tiles);
+      zgemm_dmma_persistent<2, 2><<<(unsigned)grid, 128, GEMM2_SMEM, st>>>(*b, total_tiles);
     else
-      zgemm_dmma_persistent<2, 4><<<(unsigned)grid, 256, GEMM2_SMEM, st>>>(d_descs, n, total_tiles);
+      zgemm_dmma_persistent<2, 4><<<(unsigned)grid, 256, GEMM2_SMEM, st>>>(*b, total_tiles);
     return cudaGetLastError();
   }
   switch (cls) {
-    case 0: return launch_ws<true, true>(d_descs, n, total_tiles, sms, st);
-    case 1: return launch_ws<true, false>(d_descs, n, total_tiles, sms, st);
-    case 2: return launch_ws<false, true>(d_descs, n, total_tiles, sms, st);
-    default: return launch_ws<false, false>(d_descs, n, total_tiles, sms, st);
+    case 0: return launch_ws<true, true>(b, total_tiles, sms, st);
+    case 1: return launch_ws<true, false>(b, total_tiles, sms, st);
+    case 2: return launch_ws<false, true>(b, total_tiles, sms, st);
+    default: return launch_ws<false, false>(b, total_tiles, sms, st);
   }
 }
 
-cudaError_t launch_dot_group(const DotDesc *d_descs, int n, long long total_ctas, cudaStream_t st) {
+cudaError_t launch_dot_group(const DotBatch *b, long long total_ctas, cudaStream_t st) {
   if (total_ctas <= 0) return cudaSuccess;
   static bool attr = false;
   if (!attr) {
@@ -1095,7 +1133,7 @@ cudaError_t launch_dot_group(const DotDesc *d_descs, int n, long long total_ctas
     if (e != cudaSuccess) return e;
     attr = true;
   }
-  zdot_kernel<<<(unsigned)total_ctas, DT, DOT_SMEM, st>>>(d_descs, n);
+  zdot_kernel<<<(unsigned)total_ctas, DT, DOT_SMEM, st>>>(*b);
   return cudaGetLastError();
 }
 

@@ -57,6 +57,19 @@ struct DotDesc {
 
 constexpr int kGemmBM = 64, kGemmBN = 64, kGemmBK = 8, kGemmStages = 4, kGemmThreads = 128;
 
+// A grouped launch's descriptors, passed by value as one __grid_constant__ kernel parameter
+// (≤ 32 KB of parameters per launch on sm_100).
+constexpr int kGemmBatch = 128, kDotBatch = 192;
+struct GemmBatch {
+  int n, pad;
+  GemmDesc d[kGemmBatch];
+};
+struct DotBatch {
+  int n, pad;
+  DotDesc d[kDotBatch];
+};
+static_assert(sizeof(GemmBatch) <= 32764 && sizeof(DotBatch) <= 32764, "kernel parameter limit");
+
 // GEMM descriptors carry their operand-layout class (layout.h gemm_class): 0..3 = unit-stride
 // inner index for both operands (warp-specialized kernel), 4 = generic gather kernel.
 constexpr int kGemmClasses = 5;
@@ -67,8 +80,8 @@ int gemm_variant();
 void gemm_tile_shape(int cls, int *bm, int *bn);
 
 // Grouped launches: descs in device memory (all of one layout class); grid covers the tiles.
-cudaError_t launch_gemm_group(const GemmDesc *d_descs, int n, long long total_tiles, int cls, cudaStream_t st);
-cudaError_t launch_dot_group(const DotDesc *d_descs, int n, long long total_ctas, cudaStream_t st);
+cudaError_t launch_gemm_group(const GemmBatch *b, long long total_tiles, int cls, cudaStream_t st);
+cudaError_t launch_dot_group(const DotBatch *b, long long total_ctas, cudaStream_t st);
 
 // vals[g][t] = Π_{c in comps(g)} S[slot_c][t] (component scalars)
 cudaError_t launch_finalize(int G, int Lt, const int *comp_off, const int *comp_slot,
