@@ -310,6 +310,9 @@ def main():
         "gpu_launches": launches,
         "clocks": clk,
         "sched_ms_per_step": statistics.mean(s["sched_ms"] for s in stats),
+        "breakdown_ms_per_step": {"gemm": statistics.mean(s["gemm_kernel_ms"] for s in stats),
+                                  "dot": statistics.mean(s["dot_kernel_ms"] for s in stats),
+                                  "host_enqueue": statistics.mean(s["enqueue_ms"] for s in stats)},
         "correlator_t0": [C[0].real, C[0].imag],
     }
     print(json.dumps(line), flush=True)
