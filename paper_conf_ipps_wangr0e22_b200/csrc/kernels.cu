@@ -863,7 +863,7 @@ __device__ __forceinline__ void cmac(double &sr, double &si, double2 a, double2 
   si += a.x * b.y + a.y * b.x;
 }
 
-constexpr int DOT_SMEM = (DT / 32) * 32 * 17 * 16;  // one 32×17 complex slab per warp (69.6 KB)
+constexpr int DOT_SMEM = 2 * 32 * 33 * 16;  // two 32×33 complex tiles (33.8 KB)
 
 __device__ __forceinline__ void zdot_body(const DotDesc *__restrict__ descs, int n_desc) {
   extern __shared__ __align__(16) double2 dsm[];
@@ -904,40 +904,26 @@ __device__ __forceinline__ void zdot_body(const DotDesc *__restrict__ descs, int
       const long long offB = o0 * d.sBo[0] + o1 * d.sBo[1] + o2 * d.sBo[2] + x * d.sBx;
       cmac(sr, si, A[offA], B[offB]);
     }
-  } else {
-    // transposed pair (A contiguous along x, B along y): every warp owns 32(x)×16(y) sub-tiles;
-    // A rows stay in registers (16 independent coalesced loads per lane), the B block goes
-    // through the warp's own padded smem slab (16 coalesced loads per lane), so no CTA-wide
-    // barrier and 32 loads in flight per lane.
-    double2 *Bs = dsm + (tid >> 5) * (32 * 17);
-    const int lane = tid & 31;
-    const int nx = (d.X + 31) / 32, ny = (d.Y + 15) / 16;
-    const long long nsub = Ototal * nx * ny;
-    for (long long sub = tid >> 5; sub < nsub; sub += DT / 32) {
-      const long long o = sub / (nx * ny);
-      const int rem = (int)(sub - o * nx * ny);
-      const int y0 = (rem / nx) * 16, x0 = (rem % nx) * 32;
+  } else {  // transpose tiles: A contiguous along x, B contiguous along y (32×32 smem tiles)
+    double2 (*As)[33] = reinterpret_cast<double2 (*)[33]>(dsm);
+    double2 (*Bs)[33] = reinterpret_cast<double2 (*)[33]>(dsm + 32 * 33);
+    const int ty = tid >> 5, tx = tid & 31;
+    for (long long o = 0; o < Ototal; ++o) {
       const long long o2 = o % O2, o01 = o / O2, o1 = o01 % O1, o0 = o01 / O1;
       const double2 *Ao = A + o0 * d.sAo[0] + o1 * d.sAo[1] + o2 * d.sAo[2];
       const double2 *Bo = B + o0 * d.sBo[0] + o1 * d.sBo[1] + o2 * d.sBo[2];
-      double2 a[16];
-      const int x = x0 + lane;
-#pragma unroll
-      for (int r = 0; r < 16; ++r) {
-        const int y = y0 + r;
-        a[r] = (y < d.Y && x < d.X) ? Ao[(long long)y * d.sAy + (long long)x * d.sAx] : make_double2(0.0, 0.0);
-      }
-      __syncwarp();
-#pragma unroll
-      for (int rr = 0; rr < 16; ++rr) {
-        const int xl = 2 * rr + (lane >> 4), yl = lane & 15;
-        const int xb = x0 + xl, yb = y0 + yl;
-        Bs[xl * 17 + yl] = (xb < d.X && yb < d.Y) ? Bo[(long long)xb * d.sBx + (long long)yb * d.sBy]
-                                                  : make_double2(0.0, 0.0);
-      }
-      __syncwarp();
-#pragma unroll
-      for (int r = 0; r < 16; ++r) cmac(sr, si, a[r], Bs[lane * 17 + r]);
+      for (int y0 = 0; y0 < d.Y; y0 += 32)
+        for (int x0 = 0; x0 < d.X; x0 += 32) {
+          for (int r = ty; r < 32; r += DT / 32) {
+            const int y = y0 + r, x = x0 + tx;
+            As[r][tx] = (y < d.Y && x < d.X) ? Ao[(long long)y * d.sAy + (long long)x * d.sAx] : make_double2(0, 0);
+            const int xb = x0 + r, yb = y0 + tx;
+            Bs[r][tx] = (xb < d.X && yb < d.Y) ? Bo[(long long)xb * d.sBx + (long long)yb * d.sBy] : make_double2(0, 0);
+          }
+          __syncthreads();
+          for (int r = ty; r < 32; r += DT / 32) cmac(sr, si, As[r][tx], Bs[tx][r]);
+          __syncthreads();
+        }
     }
   }
   // deterministic block reduction: xor butterfly, then warps in order
