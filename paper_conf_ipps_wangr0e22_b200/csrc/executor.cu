@@ -609,7 +609,8 @@ struct Executor::Impl {
     in.keep_inputs = c.opt.keep_inputs_resident != 0;
     {
       const char *gv = getenv("MICCO_GEMM"), *nf = getenv("MICCO_NO_FUSE");
-      in.fuse = gemm_variant() == 3 && !(nf && nf[0] == '1');  // the fused epilogue exists in v3 only
+      // the fused epilogue exists in the persistent (2, default) and warp-specialized (3) kernels
+      in.fuse = (gemm_variant() == 2 || gemm_variant() == 3) && !(nf && nf[0] == '1');
       (void)gv;
     }
     in.peer_gbs = (ndev > 1 && !dist()) || dist() ? 700 : 2500;

@@ -347,6 +347,8 @@ struct LoadCur {
 struct StoreCur {
   double2 *C;
   int sCmi, sCni, Mi, Ni, m0, n0, KTOT;
+  const double2 *D;  // fused final dot: the partner tile base (nullptr = plain GEMM)
+  long long pidx;    // first partial-sum slot of this tile
 };
 
 template <int NTH, int LPT>
@@ -390,6 +392,8 @@ __device__ __forceinline__ void decode_tile(const GemmDesc *__restrict__ descs, 
     S->sCmi = (int)d.sCmi; S->sCni = (int)d.sCni;
     S->Mi = d.Mi; S->Ni = d.Ni; S->m0 = m0; S->n0 = n0;
     S->KTOT = d.Ko * KT;
+    S->D = d.D ? d.D + t * d.sDt + mo * d.sDmo + no * d.sDno : nullptr;
+    S->pidx = (tile - d.tile_begin) * (NTH / 32);
   }
 }
 
@@ -529,19 +533,65 @@ __device__ __forceinline__ void zgemm_dmma_persistent_body(const GemmDesc *__res
     cp_async_commit();
     slot_l = (slot_l + 1 == ST2) ? 0 : slot_l + 1;
     slot_c = (slot_c + 1 == ST2) ? 0 : slot_c + 1;
+    if (S.D && kt_c + 2 == S.KTOT) {
+      // fused dot: pull this tile's partner block into L2 one k-step before the epilogue
+      const GemmDesc &dd = descs[task_c];
+      const bool mrow = dd.sDni == 1;  // contiguous runs along n (else along m, sDmi == 1)
+      const int rows = mrow ? min(BM, S.Mi - S.m0) : min(BN, S.Ni - S.n0);
+      for (int q = tid; q < rows * 8; q += NTH) {
+        const int r = q >> 3, seg = (q & 7) * 8;
+        const double2 *pp = mrow ? S.D + (long long)(S.m0 + r) * dd.sDmi + S.n0 + seg
+                                 : S.D + (long long)(S.n0 + r) * dd.sDni + S.m0 + seg;
+        asm volatile("prefetch.global.L2 [%0];\n" ::"l"(pp));
+      }
+    }
     if (++kt_c == S.KTOT) {  // tile done: write back (next tile's loads already in flight)
+      if (S.D) {
+        // fused final contraction: this warp's partial Σ C·D (no C written), 8 loads in flight
+        const GemmDesc &dd = descs[task_c];
+        const long long sDmi = dd.sDmi, sDni = dd.sDni;
+        double pr = 0.0, pim = 0.0;
 #pragma unroll
-      for (int i = 0; i < MI; ++i) {
-        const int m = S.m0 + wm * MI * 8 + i * 8 + (lane >> 2);
+        for (int i = 0; i < MI; ++i) {
+          const int m = S.m0 + wm * MI * 8 + i * 8 + (lane >> 2);
+          double2 y[NJ][2];
 #pragma unroll
-        for (int j = 0; j < NJ; ++j) {
-          const int n = S.n0 + wn * NJ * 8 + j * 8 + (lane & 3) * 2;
-          if (m < S.Mi) {
-            double2 *cp = S.C + (long long)m * S.sCmi + (long long)n * S.sCni;
-            if (n < S.Ni) cp[0] = make_double2(cr[i][j][0], ci[i][j][0]);
-            if (n + 1 < S.Ni) cp[S.sCni] = make_double2(cr[i][j][1], ci[i][j][1]);
+          for (int j = 0; j < NJ; ++j)
+#pragma unroll
+            for (int h = 0; h < 2; ++h) {
+              const int n = S.n0 + wn * NJ * 8 + j * 8 + (lane & 3) * 2 + h;
+              y[j][h] = (m < S.Mi && n < S.Ni) ? S.D[(long long)m * sDmi + (long long)n * sDni] : make_double2(0.0, 0.0);
+            }
+#pragma unroll
+          for (int j = 0; j < NJ; ++j)
+#pragma unroll
+            for (int h = 0; h < 2; ++h) {
+              pr += cr[i][j][h] * y[j][h].x - ci[i][j][h] * y[j][h].y;
+              pim += cr[i][j][h] * y[j][h].y + ci[i][j][h] * y[j][h].x;
+              cr[i][j][h] = 0.0;
+              ci[i][j][h] = 0.0;
+            }
+        }
+#pragma unroll
+        for (int off = 16; off > 0; off >>= 1) {
+          pr += __shfl_xor_sync(0xffffffffu, pr, off);
+          pim += __shfl_xor_sync(0xffffffffu, pim, off);
+        }
+        if (lane == 0) dd.part[S.pidx + warp] = make_double2(pr, pim);
+      } else {
+#pragma unroll
+        for (int i = 0; i < MI; ++i) {
+          const int m = S.m0 + wm * MI * 8 + i * 8 + (lane >> 2);
+#pragma unroll
+          for (int j = 0; j < NJ; ++j) {
+            const int n = S.n0 + wn * NJ * 8 + j * 8 + (lane & 3) * 2;
+            if (m < S.Mi) {
+              double2 *cp = S.C + (long long)m * S.sCmi + (long long)n * S.sCni;
+              if (n < S.Ni) cp[0] = make_double2(cr[i][j][0], ci[i][j][0]);
+              if (n + 1 < S.Ni) cp[S.sCni] = make_double2(cr[i][j][1], ci[i][j][1]);
+            }
+            cr[i][j][0] = cr[i][j][1] = ci[i][j][0] = ci[i][j][1] = 0.0;
           }
-          cr[i][j][0] = cr[i][j][1] = ci[i][j][0] = ci[i][j][1] = 0.0;
         }
       }
       kt_c = 0;
