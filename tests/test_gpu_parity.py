@@ -161,3 +161,17 @@ def test_c3_sampled_n256():
     """C3 meson wirings at N = 256 (the multi-meson config's tensor size), Lt = 4."""
     wl = workloads.c3_multi_meson(n_graphs=40, N=256, Lt=4, pool=4)
     check(wl.subset(list(range(12))))
+
+
+def test_multiprocess_mode_single_rank_nccl():
+    """The one-process-per-GPU path (plan replay of this rank's ops, NCCL communicator,
+    ncclAllReduce of the scalar table) with world size 1: same C(t) bit for bit."""
+    wl = workloads.c1_two_meson()
+    ref, _, _ = run_gpu(wl)
+    ctx = M.Context(dist_rank=0, dist_world=1)
+    M.load_workload(ctx, wl)
+    M.micco_set_nccl_id(ctx.h, M.micco_nccl_unique_id())
+    ctx.execute(1)
+    C = ctx.correlator()
+    ctx.close()
+    assert np.array_equal(C, ref)
