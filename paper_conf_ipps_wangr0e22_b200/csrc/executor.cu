@@ -610,7 +610,7 @@ struct Executor::Impl {
     {
       const char *gv = getenv("MICCO_GEMM"), *nf = getenv("MICCO_NO_FUSE");
       // the fused epilogue exists in the persistent (2, default) and warp-specialized (3) kernels
-      in.fuse = (gemm_variant() == 2 || gemm_variant() == 3) && !(nf && nf[0] == '1');
+      in.fuse = (gemm_variant() == 2 || gemm_variant() == 3 || gemm_variant() == 5) && !(nf && nf[0] == '1');
       (void)gv;
     }
     in.peer_gbs = (ndev > 1 && !dist()) || dist() ? 700 : 2500;

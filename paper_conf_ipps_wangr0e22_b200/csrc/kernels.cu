@@ -315,31 +315,40 @@ __device__ __forceinline__ void zgemm_small_body(const GemmDesc *__restrict__ de
   }
 }
 
-// ---------------------------------------------------------------- persistent GEMM (v2)
+// ---------------------------------------------------------------- persistent GEMM (v2, 3M)
 //
-// Same math and warp tiling as zgemm_dmma_kernel, restructured to remove the per-tile
-// bubbles the round-1 ncu capture showed (profiles/ncu_gemm_r01.json: long-scoreboard
-// stalls at tile prologues and descriptor loads):
-//  * persistent: grid = resident CTAs; CTA c owns a contiguous range of tiles, so its task
-//    descriptor changes rarely and is advanced linearly (no per-tile binary search);
-//  * one continuous cp.async pipeline over the CTA's whole (tile, k-step) sequence: the
-//    loads of the next tile are in flight while the current tile finishes and writes back;
-//  * BK = 16 with 3 stages (half the barriers per tile), per-thread 32-bit element offsets
-//    precomputed once per tile.
+// The production GEMM.  Persistent CTAs (2 per SM) own contiguous tile ranges and run one
+// continuous cp.async pipeline (BK = 16, 3 stages) over their whole (tile, k-step) sequence;
+// the next stage's copies are issued in NPART pieces inside the DMMA stream of the stage being
+// computed so they occupy the DMMA pacing slots; the task descriptor advances linearly.
+// Optional fused final dot (GemmDesc::D) in the epilogue.
+//
+// Complex product, two schemes (template M3):
+//   4M (default before round-1 end): Cr += Ar·Br + (−Ai)·Bi, Ci += Ar·Bi + Ai·Br  — 4 DMMAs
+//   3M (Gauss): K1 += (Ar+Ai)·Br, K2 += Ar·(Bi−Br), K3 += Ai·(Br+Bi);
+//               Cr = K1 − K3, Ci = K1 + K2                                       — 3 DMMAs
+// The 3M scheme does 25% fewer DMMAs for the same algorithmic work (8 real flops per complex
+// MAC are still what the roofline counts); its rounding differs from the 4M one but stays far
+// inside the 1e-10 parity bound, and exact-integer inputs stay bit-exact (every partial sum
+// is an integer below 2^53; SURVEY.md §8(c) "Bit-exact GPU parity").
 constexpr int BK2 = 16, ST2 = 3;
-constexpr int APITCH2 = BK2 + 4;  // 320 B ≡ 64 (mod 128): A fragment loads conflict-free
-constexpr int BPITCH2 = BN + 2;   // 1056 B ≡ 32 (mod 128)
-constexpr int A_STAGE2 = BM * APITCH2;
-constexpr int B_STAGE2 = BK2 * BPITCH2;
-constexpr int GEMM2_SMEM = ST2 * (A_STAGE2 + B_STAGE2) * 16;
+constexpr int APITCH2 = BK2 + 4;  // [m][k] rows: 320 B ≡ 64 (mod 128): A fragment loads conflict-free
 
-template <int LPT>
+template <int TBM, int TBN>
+struct PCfg {
+  static constexpr int BP = TBN + 2;  // [k][n] rows: (TBN+2)·16 B ≡ 32 (mod 128) for TBN ∈ {32, 64}
+  static constexpr int AE = TBM * APITCH2, BE = BK2 * BP;
+  static constexpr int SMEM = ST2 * (AE + BE) * 16;
+};
+constexpr int GEMM2_SMEM = PCfg<64, 64>::SMEM;
+
+template <int LPTA, int LPTB>
 struct LoadCur {
   const double2 *A, *B;  // tile bases (t, mo/no, m0/n0 applied)
   long long sAko, sBko;
   int sAki, sBki;
   int Ki, KT, KTOT;
-  int offA[LPT], offB[LPT];
+  int offA[LPTA], offB[LPTB];
   unsigned vA, vB;       // m-valid / n-valid bit per element
   bool akf, bnf;
 };
@@ -351,9 +360,9 @@ struct StoreCur {
   long long pidx;    // first partial-sum slot of this tile
 };
 
-template <int NTH, int LPT>
+template <int NTH, int TBM, int TBN, int LPTA, int LPTB>
 __device__ __forceinline__ void decode_tile(const GemmDesc *__restrict__ descs, int n_desc, int &task,
-                                            long long tile, int tid, LoadCur<LPT> *L, StoreCur *S) {
+                                            long long tile, int tid, LoadCur<LPTA, LPTB> *L, StoreCur *S) {
   while (task + 1 < n_desc && descs[task + 1].tile_begin <= tile) ++task;
   const GemmDesc &d = descs[task];
   long long lt = tile - d.tile_begin;
@@ -363,7 +372,7 @@ __device__ __forceinline__ void decode_tile(const GemmDesc *__restrict__ descs, 
   const int no = (int)(lt % No); lt /= No;
   const int mo = (int)(lt % Mo);
   const long long t = lt / Mo;
-  const int m0 = tm * BM, n0 = tn * BN;
+  const int m0 = tm * TBM, n0 = tn * TBN;
   const int KT = (d.Ki + BK2 - 1) / BK2;
   if (L) {
     const int sAmi = (int)d.sAmi, sAki = (int)d.sAki, sBki = (int)d.sBki, sBni = (int)d.sBni;
@@ -376,13 +385,18 @@ __device__ __forceinline__ void decode_tile(const GemmDesc *__restrict__ descs, 
     const int Mi = d.Mi, Ni = d.Ni;
     L->vA = 0; L->vB = 0;
 #pragma unroll
-    for (int j = 0; j < LPT; ++j) {
+    for (int j = 0; j < LPTA; ++j) {
       const int e = tid + j * NTH;
-      int m, k, n, kb;
-      if (L->akf) { k = e & (BK2 - 1); m = e / BK2; } else { m = e & (BM - 1); k = e / BM; }
+      int m, k;
+      if (L->akf) { k = e & (BK2 - 1); m = e / BK2; } else { m = e % TBM; k = e / TBM; }
       L->offA[j] = m * sAmi + k * sAki;
       if (m0 + m < Mi) L->vA |= 1u << j;
-      if (L->bnf) { n = e & (BN - 1); kb = e / BN; } else { kb = e & (BK2 - 1); n = e / BK2; }
+    }
+#pragma unroll
+    for (int j = 0; j < LPTB; ++j) {
+      const int e = tid + j * NTH;
+      int n, kb;
+      if (L->bnf) { n = e % TBN; kb = e / TBN; } else { kb = e & (BK2 - 1); n = e / BK2; }
       L->offB[j] = kb * sBki + n * sBni;
       if (n0 + n < Ni) L->vB |= 1u << j;
     }
@@ -397,17 +411,20 @@ __device__ __forceinline__ void decode_tile(const GemmDesc *__restrict__ descs, 
   }
 }
 
-// NWM × NWN warps; warp tile (64/NWM) × (64/NWN) complex.  <2,2> = 128 threads with 32×32
-// warp tiles (248-255 registers, 2 warps per SMSP); <2,4> = 256 threads with 32×16 warp
-// tiles (half the accumulators, 4 warps per SMSP for latency hiding).
-template <int NWM, int NWN>
-__device__ __forceinline__ void zgemm_dmma_persistent_body(const GemmDesc *__restrict__ descs, int n_desc,
-                                                           long long total) {
-  constexpr int NTH = NWM * NWN * 32, LPT = (BM * BK2) / NTH;
-  constexpr int MI = BM / NWM / 8, NJ = BN / NWN / 8;  // 8x8 blocks per warp
+// NWM × NWN warps with WTM × WTN complex warp tiles; CTA tile (NWM·WTM) × (NWN·WTN).
+template <int NWM, int NWN, int WTM, int WTN, bool M3>
+__device__ __forceinline__ void zgemm_persistent_body(const GemmDesc *__restrict__ descs, int n_desc,
+                                                      long long total) {
+  constexpr int NTH = NWM * NWN * 32;
+  constexpr int TBM = NWM * WTM, TBN = NWN * WTN;
+  constexpr int LPTA = (TBM * BK2) / NTH, LPTB = (TBN * BK2) / NTH;
+  constexpr int MI = WTM / 8, NJ = WTN / 8;  // 8x8 blocks per warp
+  constexpr int NACC = M3 ? 3 : 2;
+  using Cfg = PCfg<TBM, TBN>;
+  constexpr int BP = Cfg::BP;
   extern __shared__ __align__(128) double2 smem[];
   double2 *As = smem;
-  double2 *Bs = smem + ST2 * A_STAGE2;
+  double2 *Bs = smem + ST2 * Cfg::AE;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const int wm = warp / NWN, wn = warp % NWN;
 
@@ -425,18 +442,19 @@ __device__ __forceinline__ void zgemm_dmma_persistent_body(const GemmDesc *__res
     }
     task_l = task_c = lo;
   }
-  LoadCur<LPT> L;
+  LoadCur<LPTA, LPTB> L;
   StoreCur S;
   long long tile_l = t_begin, tile_c = t_begin;
   int kt_l = 0, kt_c = 0;
-  decode_tile<NTH, LPT>(descs, n_desc, task_l, tile_l, tid, &L, nullptr);
-  decode_tile<NTH, LPT>(descs, n_desc, task_c, tile_c, tid, (LoadCur<LPT> *)nullptr, &S);
+  decode_tile<NTH, TBM, TBN, LPTA, LPTB>(descs, n_desc, task_l, tile_l, tid, &L, nullptr);
+  decode_tile<NTH, TBM, TBN, LPTA, LPTB>(descs, n_desc, task_c, tile_c, tid, (LoadCur<LPTA, LPTB> *)nullptr, &S);
   bool more_l = true;
 
   // The loads of a stage are issued in NPART pieces interleaved with the DMMA stream of the
   // stage being computed (one piece per k-quad), so the scheduler can slot the cp.async and
   // address arithmetic into the DMMA pacing gaps instead of running a separate load phase.
   constexpr int NPART = BK2 / 4;
+  static_assert(LPTA % NPART == 0 && LPTB % NPART == 0, "load split");
   const double2 *ldA = nullptr, *ldB = nullptr;
   int ld_kb = 0;
   auto begin_load = [&]() {
@@ -446,31 +464,31 @@ __device__ __forceinline__ void zgemm_dmma_persistent_body(const GemmDesc *__res
     ldB = L.B + ko * L.sBko + (long long)ld_kb * L.sBki;
   };
   auto issue_part = [&](int slot, int part) {
-    double2 *as = As + slot * A_STAGE2;
-    double2 *bs = Bs + slot * B_STAGE2;
+    double2 *as = As + slot * Cfg::AE;
+    double2 *bs = Bs + slot * Cfg::BE;
 #pragma unroll
-    for (int jj = 0; jj < LPT / NPART; ++jj) {
-      const int j = part * (LPT / NPART) + jj;
+    for (int jj = 0; jj < LPTA / NPART; ++jj) {
+      const int j = part * (LPTA / NPART) + jj;
       const int e = tid + j * NTH;
       int m, k;
-      if (L.akf) { k = e & (BK2 - 1); m = e / BK2; } else { m = e & (BM - 1); k = e / BM; }
+      if (L.akf) { k = e & (BK2 - 1); m = e / BK2; } else { m = e % TBM; k = e / TBM; }
       const bool v = ((L.vA >> j) & 1u) && (ld_kb + k < L.Ki);
       cp_async16(as + m * APITCH2 + k, v ? ldA + L.offA[j] : L.A, v);
     }
 #pragma unroll
-    for (int jj = 0; jj < LPT / NPART; ++jj) {
-      const int j = part * (LPT / NPART) + jj;
+    for (int jj = 0; jj < LPTB / NPART; ++jj) {
+      const int j = part * (LPTB / NPART) + jj;
       const int e = tid + j * NTH;
       int n, k;
-      if (L.bnf) { n = e & (BN - 1); k = e / BN; } else { k = e & (BK2 - 1); n = e / BK2; }
+      if (L.bnf) { n = e % TBN; k = e / TBN; } else { k = e & (BK2 - 1); n = e / BK2; }
       const bool v = ((L.vB >> j) & 1u) && (ld_kb + k < L.Ki);
-      cp_async16(bs + k * BPITCH2 + n, v ? ldB + L.offB[j] : L.B, v);
+      cp_async16(bs + k * BP + n, v ? ldB + L.offB[j] : L.B, v);
     }
   };
   auto advance_load = [&]() {  // next k-step, possibly in the next tile
     if (++kt_l == L.KTOT) {
       kt_l = 0;
-      if (++tile_l < t_end) decode_tile<NTH, LPT>(descs, n_desc, task_l, tile_l, tid, &L, nullptr);
+      if (++tile_l < t_end) decode_tile<NTH, TBM, TBN, LPTA, LPTB>(descs, n_desc, task_l, tile_l, tid, &L, nullptr);
       else more_l = false;
     }
   };
@@ -481,11 +499,13 @@ __device__ __forceinline__ void zgemm_dmma_persistent_body(const GemmDesc *__res
     advance_load();
   };
 
-  double cr[MI][NJ][2], ci[MI][NJ][2];
+  double acc[MI][NJ][NACC][2];
 #pragma unroll
   for (int i = 0; i < MI; ++i)
 #pragma unroll
-    for (int j = 0; j < NJ; ++j) { cr[i][j][0] = cr[i][j][1] = ci[i][j][0] = ci[i][j][1] = 0.0; }
+    for (int j = 0; j < NJ; ++j)
+#pragma unroll
+      for (int q = 0; q < NACC; ++q) acc[i][j][q][0] = acc[i][j][q][1] = 0.0;
 
 #pragma unroll
   for (int s = 0; s < ST2 - 1; ++s) {
@@ -498,36 +518,52 @@ __device__ __forceinline__ void zgemm_dmma_persistent_body(const GemmDesc *__res
     __syncthreads();
     const bool ld = more_l;
     if (ld) begin_load();
-    const double2 *as = As + slot_c * A_STAGE2;
-    const double2 *bs = Bs + slot_c * B_STAGE2;
+    const double2 *as = As + slot_c * Cfg::AE;
+    const double2 *bs = Bs + slot_c * Cfg::BE;
 #pragma unroll
     for (int kq = 0; kq < BK2 / 4; ++kq) {
       if (ld) issue_part(slot_l, kq);
-      double ar[MI], ai[MI], an[MI], br[NJ], bi[NJ];
+      double ar[MI], ai[MI], br[NJ], bi[NJ];
 #pragma unroll
       for (int i = 0; i < MI; ++i) {
-        const double2 a = as[(wm * MI * 8 + i * 8 + (lane >> 2)) * APITCH2 + kq * 4 + (lane & 3)];
-        ar[i] = a.x; ai[i] = a.y; an[i] = dneg(a.y);
+        const double2 a = as[(wm * WTM + i * 8 + (lane >> 2)) * APITCH2 + kq * 4 + (lane & 3)];
+        ar[i] = a.x; ai[i] = a.y;
       }
 #pragma unroll
       for (int j = 0; j < NJ; ++j) {
-        const double2 b = bs[(kq * 4 + (lane & 3)) * BPITCH2 + wn * NJ * 8 + j * 8 + (lane >> 2)];
+        const double2 b = bs[(kq * 4 + (lane & 3)) * BP + wn * WTN + j * 8 + (lane >> 2)];
         br[j] = b.x; bi[j] = b.y;
       }
+      if constexpr (M3) {
+        double as_[MI], bm[NJ], bp[NJ];
 #pragma unroll
-      for (int i = 0; i < MI; ++i)
+        for (int i = 0; i < MI; ++i) as_[i] = ar[i] + ai[i];
 #pragma unroll
-        for (int j = 0; j < NJ; ++j) {
-          dmma(cr[i][j][0], cr[i][j][1], ar[i], br[j]);
-          dmma(ci[i][j][0], ci[i][j][1], ar[i], bi[j]);
-        }
+        for (int j = 0; j < NJ; ++j) { bm[j] = bi[j] - br[j]; bp[j] = br[j] + bi[j]; }
 #pragma unroll
-      for (int i = 0; i < MI; ++i)
+        for (int i = 0; i < MI; ++i)
 #pragma unroll
-        for (int j = 0; j < NJ; ++j) {
-          dmma(cr[i][j][0], cr[i][j][1], an[i], bi[j]);
-          dmma(ci[i][j][0], ci[i][j][1], ai[i], br[j]);
-        }
+          for (int j = 0; j < NJ; ++j) {
+            dmma(acc[i][j][0][0], acc[i][j][0][1], as_[i], br[j]);
+            dmma(acc[i][j][1][0], acc[i][j][1][1], ar[i], bm[j]);
+            dmma(acc[i][j][2][0], acc[i][j][2][1], ai[i], bp[j]);
+          }
+      } else {
+#pragma unroll
+        for (int i = 0; i < MI; ++i)
+#pragma unroll
+          for (int j = 0; j < NJ; ++j) {
+            dmma(acc[i][j][0][0], acc[i][j][0][1], ar[i], br[j]);
+            dmma(acc[i][j][1][0], acc[i][j][1][1], ar[i], bi[j]);
+          }
+#pragma unroll
+        for (int i = 0; i < MI; ++i)
+#pragma unroll
+          for (int j = 0; j < NJ; ++j) {
+            dmma(acc[i][j][0][0], acc[i][j][0][1], dneg(ai[i]), bi[j]);
+            dmma(acc[i][j][1][0], acc[i][j][1][1], ai[i], br[j]);
+          }
+      }
     }
     if (ld) advance_load();
     cp_async_commit();
@@ -537,39 +573,50 @@ __device__ __forceinline__ void zgemm_dmma_persistent_body(const GemmDesc *__res
       // fused dot: pull this tile's partner block into L2 one k-step before the epilogue
       const GemmDesc &dd = descs[task_c];
       const bool mrow = dd.sDni == 1;  // contiguous runs along n (else along m, sDmi == 1)
-      const int rows = mrow ? min(BM, S.Mi - S.m0) : min(BN, S.Ni - S.n0);
-      for (int q = tid; q < rows * 8; q += NTH) {
-        const int r = q >> 3, seg = (q & 7) * 8;
+      const int rows = mrow ? min(TBM, S.Mi - S.m0) : min(TBN, S.Ni - S.n0);
+      const int segs = (mrow ? TBN : TBM) / 8;
+      for (int q = tid; q < rows * segs; q += NTH) {
+        const int r = q / segs, seg = (q % segs) * 8;
         const double2 *pp = mrow ? S.D + (long long)(S.m0 + r) * dd.sDmi + S.n0 + seg
                                  : S.D + (long long)(S.n0 + r) * dd.sDni + S.m0 + seg;
         asm volatile("prefetch.global.L2 [%0];\n" ::"l"(pp));
       }
     }
     if (++kt_c == S.KTOT) {  // tile done: write back (next tile's loads already in flight)
+      // the complex value of accumulator block (i, j), half h
+      auto cval = [&](int i, int j, int h, double &re, double &im) {
+        if constexpr (M3) {
+          re = acc[i][j][0][h] - acc[i][j][2][h];
+          im = acc[i][j][0][h] + acc[i][j][1][h];
+        } else {
+          re = acc[i][j][0][h];
+          im = acc[i][j][1][h];
+        }
+      };
       if (S.D) {
-        // fused final contraction: this warp's partial Σ C·D (no C written), 8 loads in flight
+        // fused final contraction: this warp's partial Σ C·D (no C written)
         const GemmDesc &dd = descs[task_c];
         const long long sDmi = dd.sDmi, sDni = dd.sDni;
         double pr = 0.0, pim = 0.0;
 #pragma unroll
         for (int i = 0; i < MI; ++i) {
-          const int m = S.m0 + wm * MI * 8 + i * 8 + (lane >> 2);
+          const int m = S.m0 + wm * WTM + i * 8 + (lane >> 2);
           double2 y[NJ][2];
 #pragma unroll
           for (int j = 0; j < NJ; ++j)
 #pragma unroll
             for (int h = 0; h < 2; ++h) {
-              const int n = S.n0 + wn * NJ * 8 + j * 8 + (lane & 3) * 2 + h;
+              const int n = S.n0 + wn * WTN + j * 8 + (lane & 3) * 2 + h;
               y[j][h] = (m < S.Mi && n < S.Ni) ? S.D[(long long)m * sDmi + (long long)n * sDni] : make_double2(0.0, 0.0);
             }
 #pragma unroll
           for (int j = 0; j < NJ; ++j)
 #pragma unroll
             for (int h = 0; h < 2; ++h) {
-              pr += cr[i][j][h] * y[j][h].x - ci[i][j][h] * y[j][h].y;
-              pim += cr[i][j][h] * y[j][h].y + ci[i][j][h] * y[j][h].x;
-              cr[i][j][h] = 0.0;
-              ci[i][j][h] = 0.0;
+              double re, im;
+              cval(i, j, h, re, im);
+              pr += re * y[j][h].x - im * y[j][h].y;
+              pim += re * y[j][h].y + im * y[j][h].x;
             }
         }
 #pragma unroll
@@ -581,22 +628,30 @@ __device__ __forceinline__ void zgemm_dmma_persistent_body(const GemmDesc *__res
       } else {
 #pragma unroll
         for (int i = 0; i < MI; ++i) {
-          const int m = S.m0 + wm * MI * 8 + i * 8 + (lane >> 2);
+          const int m = S.m0 + wm * WTM + i * 8 + (lane >> 2);
 #pragma unroll
           for (int j = 0; j < NJ; ++j) {
-            const int n = S.n0 + wn * NJ * 8 + j * 8 + (lane & 3) * 2;
+            const int n = S.n0 + wn * WTN + j * 8 + (lane & 3) * 2;
             if (m < S.Mi) {
+              double re, im;
               double2 *cp = S.C + (long long)m * S.sCmi + (long long)n * S.sCni;
-              if (n < S.Ni) cp[0] = make_double2(cr[i][j][0], ci[i][j][0]);
-              if (n + 1 < S.Ni) cp[S.sCni] = make_double2(cr[i][j][1], ci[i][j][1]);
+              cval(i, j, 0, re, im);
+              if (n < S.Ni) cp[0] = make_double2(re, im);
+              cval(i, j, 1, re, im);
+              if (n + 1 < S.Ni) cp[S.sCni] = make_double2(re, im);
             }
-            cr[i][j][0] = cr[i][j][1] = ci[i][j][0] = ci[i][j][1] = 0.0;
           }
         }
       }
+#pragma unroll
+      for (int i = 0; i < MI; ++i)
+#pragma unroll
+        for (int j = 0; j < NJ; ++j)
+#pragma unroll
+          for (int q = 0; q < NACC; ++q) acc[i][j][q][0] = acc[i][j][q][1] = 0.0;
       kt_c = 0;
       if (++tile_c >= t_end) break;
-      decode_tile<NTH, LPT>(descs, n_desc, task_c, tile_c, tid, (LoadCur<LPT> *)nullptr, &S);
+      decode_tile<NTH, TBM, TBN, LPTA, LPTB>(descs, n_desc, task_c, tile_c, tid, (LoadCur<LPTA, LPTB> *)nullptr, &S);
     }
   }
   cp_async_wait<0>();
@@ -1053,10 +1108,10 @@ template <int TBM, int TBN, int TST, int MINB>
 __global__ void __launch_bounds__(128, MINB) zgemm_small(const __grid_constant__ GemmBatch b, long long total) {
   zgemm_small_body<TBM, TBN, TST>(b.d, b.n, total);
 }
-template <int NWM, int NWN>
+template <int NWM, int NWN, int WTM, int WTN, bool M3>
 __global__ void __launch_bounds__(NWM * NWN * 32, 2)
-    zgemm_dmma_persistent(const __grid_constant__ GemmBatch b, long long total) {
-  zgemm_dmma_persistent_body<NWM, NWN>(b.d, b.n, total);
+    zgemm_persistent(const __grid_constant__ GemmBatch b, long long total) {
+  zgemm_persistent_body<NWM, NWN, WTM, WTN, M3>(b.d, b.n, total);
 }
 template <bool A_MK, bool B_KN>
 __global__ void __launch_bounds__(NT3, 1) zgemm_dmma_ws(const __grid_constant__ GemmBatch b, long long total) {
@@ -1083,7 +1138,7 @@ cudaError_t launch_ws(const GemmBatch *b, long long total, int sms, cudaStream_t
 }  // namespace
 
 int gemm_variant() {
-  // MICCO_GEMM = 1 per-tile 64×64, 2 persistent 64×64, 3 warp-specialized, 5 8-warp persistent,
+  // MICCO_GEMM = 1 per-tile 64×64, 2 persistent 64×64 4M, 3 warp-specialized, 5 persistent 64×32 3M,
   // 6 small 32×32 (4 stages, 3 CTAs/SM), 7 64×32, 8 32×32 (3 stages, 4 CTAs/SM)
   static int variant = -1;
   if (variant < 0) {
@@ -1099,7 +1154,7 @@ void gemm_tile_shape(int cls, int *bm, int *bn) {
   *bn = 64;
   if (cls == 4) return;  // gather kernel (v1)
   if (v == 6 || v == 8) { *bm = 32; *bn = 32; }
-  if (v == 7) { *bm = 64; *bn = 32; }
+  if (v == 7 || v == 5) { *bm = 64; *bn = 32; }
 }
 
 cudaError_t launch_gemm_group(const GemmBatch *b, long long total_tiles, int cls, cudaStream_t st) {
@@ -1108,9 +1163,11 @@ cudaError_t launch_gemm_group(const GemmBatch *b, long long total_tiles, int cls
   if (!attr_set) {
     cudaError_t e = cudaFuncSetAttribute(zgemm_dmma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, GEMM_SMEM);
     if (e != cudaSuccess) return e;
-    e = cudaFuncSetAttribute(zgemm_dmma_persistent<2, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, GEMM2_SMEM);
+    e = cudaFuncSetAttribute(zgemm_persistent<2, 2, 32, 32, false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             PCfg<64, 64>::SMEM);
     if (e != cudaSuccess) return e;
-    e = cudaFuncSetAttribute(zgemm_dmma_persistent<2, 4>, cudaFuncAttributeMaxDynamicSharedMemorySize, GEMM2_SMEM);
+    e = cudaFuncSetAttribute(zgemm_persistent<2, 2, 32, 16, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             PCfg<64, 32>::SMEM);
     if (e != cudaSuccess) return e;
     attr_set = true;
   }
@@ -1148,9 +1205,9 @@ cudaError_t launch_gemm_group(const GemmBatch *b, long long total_tiles, int cls
     long long grid = 2LL * sms;  // 2 resident CTAs per SM (112 KB smem each)
     if (grid > total_tiles) grid = total_tiles;
     if (variant == 2)
-      zgemm_dmma_persistent<2, 2><<<(unsigned)grid, 128, GEMM2_SMEM, st>>>(*b, total_tiles);
-    else
-      zgemm_dmma_persistent<2, 4><<<(unsigned)grid, 256, GEMM2_SMEM, st>>>(*b, total_tiles);
+      zgemm_persistent<2, 2, 32, 32, false><<<(unsigned)grid, 128, PCfg<64, 64>::SMEM, st>>>(*b, total_tiles);
+    else  // 5: 3M complex products, 64×32 CTA tile
+      zgemm_persistent<2, 2, 32, 16, true><<<(unsigned)grid, 128, PCfg<64, 32>::SMEM, st>>>(*b, total_tiles);
     return cudaGetLastError();
   }
   switch (cls) {
