@@ -185,7 +185,9 @@ typedef struct {
   double dot_bytes;            /* algorithmic bytes read by the dot/trace tasks executed */
   double enqueue_ms;           /* host time spent replaying the plan (issuing copies/kernels) */
   int32_t host_pinned;         /* 1 if every node tensor lives in page-locked host memory */
-  int32_t reserved0;
+  int32_t gemm_3m;             /* 1 if the GEMMs used 3 real DMMA products per complex MAC (Gauss) */
+  double gemm_dmma_flops;      /* flops actually executed on the DMMA pipe by the GEMMs
+                                  (= gemm_flops, or 6/8 of it with the 3M scheme) */
 } micco_stats;
 
 MICCO_API micco_status micco_get_stats(const micco_ctx *ctx, micco_stats *out);

@@ -261,3 +261,70 @@ def tiny_random(seed: int = 7, n_graphs: int = 20, N: int = 3, Lt: int = 2, mode
         order = [int(x) for x in rng.permutation(len(edges))]
         graphs.append(GraphSpec(inst, edges, order, _rand_coef(rng)))
     return Workload("tiny_random", Lt, seed, mode, nodes, graphs, {"N": N})
+
+
+# ---------------------------------------------------------------- C5
+
+
+def c5_mixed(n_combos: int = 4, Nb: int = 64, Nm: int = 256, Lt: int = 64, pool: int = 4,
+             meson_graphs: int = 64, seed: int = 5, mode: int = MODE_UNIFORM) -> Workload:
+    """C5 (configs[4]): memory-oversubscribed mixed meson/baryon set.
+
+    Baryon part: connected two-baryon matchings only (S1 shares 1 or 2 legs with each
+    source), with a forced first step S1 × (the source it shares exactly ONE leg with) —
+    a rank-4 intermediate of Nb^4·Lt complex (16 GiB at Nb = 64, Lt = 64), shared by every
+    graph with the same (S1, source, leg pair) — then that rank-4 tensor × S1's two-leg
+    partner over 2 legs (rank 3), then the final rank-3 dot with S2.  Consumers of one
+    rank-4 tensor are spread over the whole graph stream so it stays live.
+    Meson part: C3-style 3-meson wirings at Nm, interleaved with the baryon graphs.
+    Each context has one Lt (nodes may differ in N)."""
+    rng = np.random.default_rng(seed)
+    nodes = [NodeSpec(3, Nb, 50000 + i) for i in range(2 * pool)]
+    mbase = len(nodes)
+    mpool = max(3, pool)
+    nodes += [NodeSpec(2, Nm, 51000 + i) for i in range(2 * mpool)]
+    allm = two_baryon_matchings()
+    connected = [mi for mi, m in enumerate(allm) if sum(1 for s, r in m if s < 3 and r < 3) in (1, 2)]
+    baryon = []
+    seen = set()
+    while len(seen) < n_combos:
+        S = tuple(int(x) for x in rng.choice(pool, 2, replace=False))
+        R = tuple(pool + int(x) for x in rng.choice(pool, 2, replace=False))
+        if (S, R) in seen:
+            continue
+        seen.add((S, R))
+        for mi in connected:
+            m = allm[mi]
+            inst = [S[0], S[1], R[0], R[1]]
+            edges = [(sl // 3, sl % 3, 2 + rl // 3, rl % 3) for sl, rl in m]
+
+            def between(a, b):
+                return [i for i, (u, _, v, _) in enumerate(edges) if {u, v} == {a, b}]
+            one = 2 if len(between(0, 2)) == 1 else 3      # S1's single-leg partner
+            two = 5 - one                                  # S1's two-leg partner
+            first, second = between(0, one), between(0, two)
+            rest = [i for i in range(len(edges)) if i not in first and i not in second]
+            baryon.append(GraphSpec(inst, edges, first + second + rest, _rand_coef(rng)))
+    rng.shuffle(baryon)
+    perms = list(itertools.permutations(range(3)))
+    mesons = []
+    while len(mesons) < meson_graphs:
+        Sm = [mbase + int(x) for x in rng.choice(mpool, 3, replace=False)]
+        Rm = [mbase + mpool + int(x) for x in rng.choice(mpool, 3, replace=False)]
+        pi = perms[int(rng.integers(0, 6))]
+        rho = perms[int(rng.integers(0, 6))]
+        edges = []
+        for a in range(3):
+            edges.append((a, 1, 3 + pi[a], 0))
+            edges.append((a, 0, 3 + rho[a], 1))
+        mesons.append(GraphSpec(Sm + Rm, edges, cycle_chain_order(6, edges), _rand_coef(rng)))
+    graphs = []
+    step = max(1, len(baryon) // max(1, len(mesons)))
+    mi = 0
+    for i, g in enumerate(baryon):
+        graphs.append(g)
+        if i % step == step - 1 and mi < len(mesons):
+            graphs.append(mesons[mi])
+            mi += 1
+    graphs += mesons[mi:]
+    return Workload("c5_mixed", Lt, seed, mode, nodes, graphs, {"Nb": Nb, "Nm": Nm})

@@ -440,6 +440,9 @@ struct Executor::Impl {
       }
       l.gemm.push_back(d);
       st.gemm_flops += tk.flops;
+      const bool m3 = gemm_uses_3m(d.cls);
+      st.gemm_dmma_flops += m3 ? tk.flops * 0.75 : tk.flops;
+      if (m3) st.gemm_3m = 1;
     } else {
       DotLayout L;
       double2 *pb = nullptr;

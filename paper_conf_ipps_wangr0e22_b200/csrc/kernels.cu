@@ -1138,12 +1138,13 @@ cudaError_t launch_ws(const GemmBatch *b, long long total, int sms, cudaStream_t
 }  // namespace
 
 int gemm_variant() {
-  // MICCO_GEMM = 1 per-tile 64×64, 2 persistent 64×64 4M, 3 warp-specialized, 5 persistent 64×32 3M,
+  // MICCO_GEMM = 1 per-tile 64×64, 2 persistent 64×64 4M, 3 warp-specialized, 5 persistent 64×32 3M
+  // (default: 19.7k vs 18.8k graphs/s for 2 on the bench workload, profiles/bench_r01_v4.json),
   // 6 small 32×32 (4 stages, 3 CTAs/SM), 7 64×32, 8 32×32 (3 stages, 4 CTAs/SM)
   static int variant = -1;
   if (variant < 0) {
     const char *e = getenv("MICCO_GEMM");
-    variant = (e && e[0] >= '1' && e[0] <= '8' && e[0] != '4') ? e[0] - '0' : 2;
+    variant = (e && e[0] >= '1' && e[0] <= '8' && e[0] != '4') ? e[0] - '0' : 5;
   }
   return variant;
 }
@@ -1156,6 +1157,8 @@ void gemm_tile_shape(int cls, int *bm, int *bn) {
   if (v == 6 || v == 8) { *bm = 32; *bn = 32; }
   if (v == 7 || v == 5) { *bm = 64; *bn = 32; }
 }
+
+bool gemm_uses_3m(int cls) { return cls != 4 && gemm_variant() == 5; }
 
 cudaError_t launch_gemm_group(const GemmBatch *b, long long total_tiles, int cls, cudaStream_t st) {
   static bool attr_set = false;  // per process; the attribute is per-function, all devices

@@ -78,6 +78,7 @@ constexpr int kGemmClasses = 5;
 // elements) for a layout class; tilesM/tilesN of a descriptor must use this shape.
 int gemm_variant();
 void gemm_tile_shape(int cls, int *bm, int *bn);
+bool gemm_uses_3m(int cls);  // 3 DMMA products per complex MAC for this layout class
 
 // Grouped launches: descs in device memory (all of one layout class); grid covers the tiles.
 cudaError_t launch_gemm_group(const GemmBatch *b, long long total_tiles, int cls, cudaStream_t st);

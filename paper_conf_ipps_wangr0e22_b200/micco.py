@@ -54,7 +54,8 @@ class micco_stats(ctypes.Structure):
                 ("gemm_kernel_ms", ctypes.c_double), ("dot_kernel_ms", ctypes.c_double),
                 ("gemm_launches", ctypes.c_int64), ("dot_launches", ctypes.c_int64),
                 ("gemm_flops", ctypes.c_double), ("dot_bytes", ctypes.c_double),
-                ("enqueue_ms", ctypes.c_double), ("host_pinned", ctypes.c_int32), ("reserved0", ctypes.c_int32)]
+                ("enqueue_ms", ctypes.c_double), ("host_pinned", ctypes.c_int32), ("gemm_3m", ctypes.c_int32),
+                ("gemm_dmma_flops", ctypes.c_double)]
 
     def as_dict(self) -> Dict:
         d = {}
