@@ -317,7 +317,7 @@ __device__ __forceinline__ void zgemm_small_body(const GemmDesc *__restrict__ de
 
 // ---------------------------------------------------------------- persistent GEMM (v2, 3M)
 //
-// The production GEMM.  Persistent CTAs (2 per SM) own contiguous tile ranges and run one
+// The production GEMM.  Persistent CTAs (2 per SM) take every G-th tile and run one
 // continuous cp.async pipeline (BK = 16, 3 stages) over their whole (tile, k-step) sequence;
 // the next stage's copies are issued in NPART pieces inside the DMMA stream of the stage being
 // computed so they occupy the DMMA pacing slots; the task descriptor advances linearly.
@@ -428,10 +428,11 @@ __device__ __forceinline__ void zgemm_persistent_body(const GemmDesc *__restrict
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const int wm = warp / NWN, wn = warp % NWN;
 
-  const long long per = total / gridDim.x, rem = total % gridDim.x;
-  const long long t_begin = blockIdx.x * per + min((long long)blockIdx.x, rem);
-  const long long t_end = t_begin + per + ((long long)blockIdx.x < rem ? 1 : 0);
-  if (t_begin >= t_end) return;
+  // CTA c takes tiles c, c + G, c + 2G, ...: the CTAs running at any moment work on
+  // neighbouring tiles (the same slices), so each A/B block is fetched from DRAM once and
+  // served to the other CTAs from L2 (contiguous per-CTA ranges doubled the DRAM reads)
+  const long long G = gridDim.x, t_begin = blockIdx.x;
+  if (t_begin >= total) return;
 
   int task_l = 0, task_c = 0;
   {  // first task by binary search, then linear advance
@@ -488,7 +489,7 @@ __device__ __forceinline__ void zgemm_persistent_body(const GemmDesc *__restrict
   auto advance_load = [&]() {  // next k-step, possibly in the next tile
     if (++kt_l == L.KTOT) {
       kt_l = 0;
-      if (++tile_l < t_end) decode_tile<NTH, TBM, TBN, LPTA, LPTB>(descs, n_desc, task_l, tile_l, tid, &L, nullptr);
+      if ((tile_l += G) < total) decode_tile<NTH, TBM, TBN, LPTA, LPTB>(descs, n_desc, task_l, tile_l, tid, &L, nullptr);
       else more_l = false;
     }
   };
@@ -650,7 +651,7 @@ __device__ __forceinline__ void zgemm_persistent_body(const GemmDesc *__restrict
 #pragma unroll
           for (int q = 0; q < NACC; ++q) acc[i][j][q][0] = acc[i][j][q][1] = 0.0;
       kt_c = 0;
-      if (++tile_c >= t_end) break;
+      if ((tile_c += G) >= total) break;
       decode_tile<NTH, TBM, TBN, LPTA, LPTB>(descs, n_desc, task_c, tile_c, tid, (LoadCur<LPTA, LPTB> *)nullptr, &S);
     }
   }
