@@ -175,3 +175,17 @@ def test_multiprocess_mode_single_rank_nccl():
     C = ctx.correlator()
     ctx.close()
     assert np.array_equal(C, ref)
+
+
+def test_c5_mixed_oversubscribed():
+    """C5 shape, scaled down: rank-4 baryon intermediates (forced c = 1 first step) mixed
+    with 3-meson graphs (different N in one context), on 2 logical GPUs with a budget a
+    few rank-4 tensors deep — evictions, D2H spills and peer copies — against the oracle."""
+    wl = workloads.c5_mixed(n_combos=1, Nb=6, Nm=10, Lt=2, pool=2, meson_graphs=12)
+    r4_bytes = 6 ** 4 * 2 * 16
+    C, vals, st = run_gpu(wl, 2, [1, 1, 1], mem_budget_bytes=6 * r4_bytes, window_graphs=32)
+    Co, valso = oracle.correlator(wl, return_values=True)
+    assert rel_err(C, Co) <= TOL
+    assert st["evictions"] > 0 and st["bytes_d2h"] > 0 and st["bytes_p2p"] > 0, st
+    ref, _, _ = run_gpu(wl, 1)
+    assert np.array_equal(C, ref)

@@ -85,3 +85,18 @@ def test_c4_matchings():
     assert len(wl.graphs) == 1440
     for G in wl.graphs[:100]:
         _valid_matching(wl, G)
+
+
+def test_c5_structure():
+    wl = workloads.c5_mixed(n_combos=1, Nb=3, Nm=4, Lt=1, pool=2, meson_graphs=6)
+    ranks = collections.Counter(n.rank for n in wl.nodes)
+    assert ranks[2] > 0 and ranks[3] > 0
+    baryon = [G for G in wl.graphs if wl.nodes[G.inst[0]].rank == 3]
+    assert len(baryon) == 648  # connected two-baryon matchings only
+    for G in baryon[:50]:
+        _valid_matching(wl, G)
+        # the first contracted pair is S1 with a source sharing exactly one leg (rank-4 step)
+        u, _, v, _ = G.edges[G.order[0]]
+        partner = v if u == 0 else u
+        shared = sum(1 for (a, _, b, _) in G.edges if {a, b} == {0, partner})
+        assert shared == 1
