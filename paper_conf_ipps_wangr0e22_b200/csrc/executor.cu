@@ -613,7 +613,8 @@ struct Executor::Impl {
     {
       const char *gv = getenv("MICCO_GEMM"), *nf = getenv("MICCO_NO_FUSE");
       // the fused epilogue exists in the persistent (2, default) and warp-specialized (3) kernels
-      in.fuse = (gemm_variant() == 2 || gemm_variant() == 3 || gemm_variant() == 5) && !(nf && nf[0] == '1');
+      const int gv2 = gemm_variant();
+      in.fuse = (gv2 == 2 || gv2 == 3 || gv2 == 5) && !(nf && nf[0] == '1');  // 4 warps per CTA
       (void)gv;
     }
     in.peer_gbs = (ndev > 1 && !dist()) || dist() ? 700 : 2500;

@@ -1114,6 +1114,11 @@ __global__ void __launch_bounds__(NWM * NWN * 32, 2)
     zgemm_persistent(const __grid_constant__ GemmBatch b, long long total) {
   zgemm_persistent_body<NWM, NWN, WTM, WTN, M3>(b.d, b.n, total);
 }
+template <int NWM, int NWN, int WTM, int WTN, bool M3>
+__global__ void __launch_bounds__(NWM * NWN * 32, 1)
+    zgemm_persistent1(const __grid_constant__ GemmBatch b, long long total) {
+  zgemm_persistent_body<NWM, NWN, WTM, WTN, M3>(b.d, b.n, total);
+}
 template <bool A_MK, bool B_KN>
 __global__ void __launch_bounds__(NT3, 1) zgemm_dmma_ws(const __grid_constant__ GemmBatch b, long long total) {
   zgemm_dmma_ws_body<A_MK, B_KN>(b.d, b.n, total);
@@ -1145,7 +1150,7 @@ int gemm_variant() {
   static int variant = -1;
   if (variant < 0) {
     const char *e = getenv("MICCO_GEMM");
-    variant = (e && e[0] >= '1' && e[0] <= '8' && e[0] != '4') ? e[0] - '0' : 5;
+    variant = (e && e[0] >= '1' && e[0] <= '8') ? e[0] - '0' : 5;
   }
   return variant;
 }
@@ -1159,7 +1164,7 @@ void gemm_tile_shape(int cls, int *bm, int *bn) {
   if (v == 7 || v == 5) { *bm = 64; *bn = 32; }
 }
 
-bool gemm_uses_3m(int cls) { return cls != 4 && gemm_variant() == 5; }
+bool gemm_uses_3m(int cls) { return cls != 4 && (gemm_variant() == 5 || gemm_variant() == 4); }
 
 cudaError_t launch_gemm_group(const GemmBatch *b, long long total_tiles, int cls, cudaStream_t st) {
   static bool attr_set = false;  // per process; the attribute is per-function, all devices
@@ -1203,6 +1208,18 @@ cudaError_t launch_gemm_group(const GemmBatch *b, long long total_tiles, int cls
       if (!a8) { cudaFuncSetAttribute(zgemm_small<32, 32, 3, 4>, cudaFuncAttributeMaxDynamicSharedMemorySize, C8::SMEM); a8 = true; }
       zgemm_small<32, 32, 3, 4><<<(unsigned)grid, 128, C8::SMEM, st>>>(*b, total_tiles);
     }
+    return cudaGetLastError();
+  }
+  if (variant == 4) {  // 3M, 8 warps of 32×16 on a 64×64 tile, one CTA per SM (255 registers)
+    static bool a4 = false;
+    if (!a4) {
+      cudaFuncSetAttribute(zgemm_persistent1<2, 4, 32, 16, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                           PCfg<64, 64>::SMEM);
+      a4 = true;
+    }
+    long long grid = sms;
+    if (grid > total_tiles) grid = total_tiles;
+    zgemm_persistent1<2, 4, 32, 16, true><<<(unsigned)grid, 256, PCfg<64, 64>::SMEM, st>>>(*b, total_tiles);
     return cudaGetLastError();
   }
   if (variant == 2 || variant == 5) {
