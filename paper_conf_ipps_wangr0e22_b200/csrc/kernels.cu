@@ -521,48 +521,64 @@ __device__ __forceinline__ void zgemm_persistent_body(const GemmDesc *__restrict
     if (ld) begin_load();
     const double2 *as = As + slot_c * Cfg::AE;
     const double2 *bs = Bs + slot_c * Cfg::BE;
-#pragma unroll
-    for (int kq = 0; kq < BK2 / 4; ++kq) {
-      if (ld) issue_part(slot_l, kq);
-      double ar[MI], ai[MI], br[NJ], bi[NJ];
+    // Fragments are double-buffered inside the stage: the LDS (and, for 3M, the operand
+    // sums on the FP64 pipe) of k-quad q+1 are issued before the DMMAs of q, so neither
+    // the shared-memory latency nor a DADD waiting behind DMMAs sits in front of them.
+    constexpr int FA = M3 ? 3 : 2, FB = M3 ? 3 : 2;
+    double fa[2][MI][FA], fb[2][NJ][FB];
+    auto load_frag = [&](int buf, int kq) {
 #pragma unroll
       for (int i = 0; i < MI; ++i) {
         const double2 a = as[(wm * WTM + i * 8 + (lane >> 2)) * APITCH2 + kq * 4 + (lane & 3)];
-        ar[i] = a.x; ai[i] = a.y;
+        fa[buf][i][0] = a.x;
+        fa[buf][i][1] = a.y;
+        if constexpr (M3) fa[buf][i][2] = a.x + a.y;  // Ar + Ai
       }
 #pragma unroll
       for (int j = 0; j < NJ; ++j) {
         const double2 b = bs[(kq * 4 + (lane & 3)) * BP + wn * WTN + j * 8 + (lane >> 2)];
-        br[j] = b.x; bi[j] = b.y;
+        fb[buf][j][0] = b.x;
+        fb[buf][j][1] = b.y;
+        if constexpr (M3) {
+          fb[buf][j][1] = b.y - b.x;  // Bi − Br
+          fb[buf][j][2] = b.x + b.y;  // Br + Bi
+        }
+      }
+    };
+    // (4M keeps a single buffer: its 128 accumulator registers leave no room for a second)
+    if constexpr (M3) load_frag(0, 0);
+#pragma unroll
+    for (int kq = 0; kq < BK2 / 4; ++kq) {
+      if (ld) issue_part(slot_l, kq);
+      const int cur = M3 ? (kq & 1) : 0;
+      if constexpr (M3) {
+        if (kq + 1 < BK2 / 4) load_frag(cur ^ 1, kq + 1);
+      } else {
+        load_frag(0, kq);
       }
       if constexpr (M3) {
-        double as_[MI], bm[NJ], bp[NJ];
-#pragma unroll
-        for (int i = 0; i < MI; ++i) as_[i] = ar[i] + ai[i];
-#pragma unroll
-        for (int j = 0; j < NJ; ++j) { bm[j] = bi[j] - br[j]; bp[j] = br[j] + bi[j]; }
 #pragma unroll
         for (int i = 0; i < MI; ++i)
 #pragma unroll
           for (int j = 0; j < NJ; ++j) {
-            dmma(acc[i][j][0][0], acc[i][j][0][1], as_[i], br[j]);
-            dmma(acc[i][j][1][0], acc[i][j][1][1], ar[i], bm[j]);
-            dmma(acc[i][j][2][0], acc[i][j][2][1], ai[i], bp[j]);
+            dmma(acc[i][j][0][0], acc[i][j][0][1], fa[cur][i][2], fb[cur][j][0]);  // (Ar+Ai)·Br
+            dmma(acc[i][j][1][0], acc[i][j][1][1], fa[cur][i][0], fb[cur][j][1]);  // Ar·(Bi−Br)
+            dmma(acc[i][j][2][0], acc[i][j][2][1], fa[cur][i][1], fb[cur][j][2]);  // Ai·(Br+Bi)
           }
       } else {
 #pragma unroll
         for (int i = 0; i < MI; ++i)
 #pragma unroll
           for (int j = 0; j < NJ; ++j) {
-            dmma(acc[i][j][0][0], acc[i][j][0][1], ar[i], br[j]);
-            dmma(acc[i][j][1][0], acc[i][j][1][1], ar[i], bi[j]);
+            dmma(acc[i][j][0][0], acc[i][j][0][1], fa[cur][i][0], fb[cur][j][0]);
+            dmma(acc[i][j][1][0], acc[i][j][1][1], fa[cur][i][0], fb[cur][j][1]);
           }
 #pragma unroll
         for (int i = 0; i < MI; ++i)
 #pragma unroll
           for (int j = 0; j < NJ; ++j) {
-            dmma(acc[i][j][0][0], acc[i][j][0][1], dneg(ai[i]), bi[j]);
-            dmma(acc[i][j][1][0], acc[i][j][1][1], ai[i], br[j]);
+            dmma(acc[i][j][0][0], acc[i][j][0][1], dneg(fa[cur][i][1]), fb[cur][j][1]);
+            dmma(acc[i][j][1][0], acc[i][j][1][1], fa[cur][i][1], fb[cur][j][0]);
           }
       }
     }
