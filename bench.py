@@ -46,6 +46,8 @@ def parse():
     ap.add_argument("--steps", type=int, default=5)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="micco", choices=["micco", "reference"])
+    ap.add_argument("--config", default="c2", choices=["c2", "c3", "c4"],
+                    help="c2 = BASELINE configs[1] (the headline); c3 / c4 = configs[2] / [3] shapes")
     ap.add_argument("--graphs", type=int, default=10000, help="graphs per GPU (weak scaling)")
     ap.add_argument("--N", type=int, default=128)
     ap.add_argument("--Lt", type=int, default=64)
@@ -108,6 +110,10 @@ class Clocks:
 
 def c2_workload(args, world):
     from micco_inputs import workloads
+    if args.config == "c3":  # multi-meson: N = 256, Lt = 128 (BASELINE configs[2])
+        return workloads.c3_multi_meson(n_graphs=args.graphs * world, N=256, Lt=128)
+    if args.config == "c4":  # two-baryon: rank-3 N = 64, Lt = 64 (configs[3]); graphs = combos × 720
+        return workloads.c4_two_baryon(n_combos=max(1, args.graphs * world // 720), N=64, Lt=64, order="greedy")
     return workloads.c2_meson_set(n_graphs=args.graphs * world, N=args.N, Lt=args.Lt, rate=args.rate,
                                   dist=args.dist, seed=2)
 
@@ -290,8 +296,10 @@ def main():
         "metric": "contraction graphs/s", "value": value, "unit": "graphs/s", "n_gpus": world,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
         "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-        "config": {"workload": wl.name, "graphs": G, "graphs_per_gpu": args.graphs, "N": args.N, "Lt": args.Lt,
-                   "rate": args.rate, "dist": args.dist, "policy": args.policy,
+        "config": {"workload": wl.name, "graphs": G, "graphs_per_gpu": args.graphs,
+                   "N": wl.meta.get("N", args.N), "Lt": wl.Lt,
+                   "rate": args.rate if args.config == "c2" else None,
+                   "dist": args.dist if args.config == "c2" else None, "policy": args.policy,
                    "parallelism": f"task-parallel x{world} (MICCO scheduler)",
                    "l2": "inputs (node tensors) larger than L2; no flush",
                    "unique_gemms": s0["n_gemm"], "unique_dots": s0["n_dot"], "dedup_hits": s0["dedup_hits"],
