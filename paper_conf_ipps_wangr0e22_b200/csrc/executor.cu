@@ -177,6 +177,7 @@ struct Executor::Impl {
   // results on device 0
   double2 *d_vals = nullptr;
   size_t vals_elems = 0;
+  int vals_dev = 0;
   double2 *h_corr = nullptr;
   int64_t launches = 0;
   bool dist() const { return c.opt.dist_world > 0; }
@@ -197,7 +198,7 @@ struct Executor::Impl {
       d.sync_events.destroy();
       d.timing_events.destroy();
     }
-    if (d_vals) { cudaSetDevice(devs.empty() ? 0 : devs[0].dev); cudaFree(d_vals); d_vals = nullptr; }
+    if (d_vals) { cudaSetDevice(vals_dev); cudaFree(d_vals); d_vals = nullptr; }
     if (h_corr) { cudaFreeHost(h_corr); h_corr = nullptr; }
     if (comm && nccl().ok) nccl().CommDestroy(comm);
     comm = nullptr;
@@ -611,11 +612,9 @@ struct Executor::Impl {
     in.window_graphs = c.opt.window_graphs;
     in.keep_inputs = c.opt.keep_inputs_resident != 0;
     {
-      const char *gv = getenv("MICCO_GEMM"), *nf = getenv("MICCO_NO_FUSE");
+      const char *nf = getenv("MICCO_NO_FUSE");
       // the fused epilogue exists in the persistent (2, default) and warp-specialized (3) kernels
-      const int gv2 = gemm_variant();
-      in.fuse = (gv2 == 2 || gv2 == 3 || gv2 == 5) && !(nf && nf[0] == '1');  // 4 warps per CTA
-      (void)gv;
+      in.fuse = gemm_fused_dot_ok() && !(nf && nf[0] == '1');
     }
     in.peer_gbs = (ndev > 1 && !dist()) || dist() ? 700 : 2500;
     in.host_gbs = 55;
@@ -732,6 +731,7 @@ struct Executor::Impl {
       if (d_vals) CK(cudaFree(d_vals));
       CK(cudaMalloc((void **)&d_vals, (size_t)G * c.Lt * sizeof(double2)));
       vals_elems = (size_t)G * c.Lt;
+      vals_dev = H.dev;
     }
     if (!h_corr) CK(cudaHostAlloc((void **)&h_corr, 1 << 20, cudaHostAllocPortable));
     double2 *d_corr = alloc(H, (int64_t)c.Lt * 16);

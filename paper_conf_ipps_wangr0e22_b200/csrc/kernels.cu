@@ -176,145 +176,6 @@ __device__ __forceinline__ void zgemm_dmma_kernel_body(const GemmDesc *__restric
   }
 }
 
-// ---------------------------------------------------------------- small-tile GEMM (v6)
-//
-// Latency hidden by warp parallelism instead of ILP: the configuration cuBLAS picks for
-// ZGEMM on this part (ncu of cuBLAS: cutlass_80_tensorop_z884gemm_32x32_16x4, 128 threads,
-// 92 registers, 3 CTAs/SM → DMMA pipe 99.5% active; profiles/ncu_cublas_r01.txt).  CTA tile
-// TBM×TBN complex, 4 warps of (TBM/2)×(TBN/2), BK 16, TST-stage cp.async ring, one tile
-// per CTA (many resident CTAs per SM overlap each other's prologue/epilogue).
-template <int TBM, int TBN, int TST>
-struct SmallCfg {
-  static constexpr int BKs = 16;
-  static constexpr int AP = BKs + 4;   // [m][k] rows: 320 B ≡ 64 (mod 128)
-  static constexpr int BP = TBN + 2;   // [k][n] rows: (TBN+2)·16 B; TBN = 32 → 544 ≡ 32 (mod 128)
-  static constexpr int AE = TBM * AP, BE = BKs * BP;
-  static constexpr int SMEM = TST * (AE + BE) * 16;
-  static constexpr int MI = TBM / 2 / 8, NJ = TBN / 2 / 8;  // 8x8 blocks per warp
-};
-
-template <int TBM, int TBN, int TST>
-__device__ __forceinline__ void zgemm_small_body(const GemmDesc *__restrict__ descs, int n_desc, long long total) {
-  using Cfg = SmallCfg<TBM, TBN, TST>;
-  constexpr int BKs = Cfg::BKs, AP = Cfg::AP, BP = Cfg::BP, MI = Cfg::MI, NJ = Cfg::NJ;
-  extern __shared__ __align__(128) double2 smem[];
-  double2 *As = smem;
-  double2 *Bs = smem + TST * Cfg::AE;
-  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  const int wm = warp >> 1, wn = warp & 1;
-  const long long tile = blockIdx.x;
-  if (tile >= total) return;
-  int lo = 0, hi = n_desc - 1;
-  while (lo < hi) {
-    int mid = (lo + hi + 1) >> 1;
-    if (descs[mid].tile_begin <= tile) lo = mid; else hi = mid - 1;
-  }
-  const GemmDesc &d = descs[lo];
-  long long lt = tile - d.tile_begin;
-  const int tilesN = d.tilesN, tilesM = d.tilesM;
-  const int tn = (int)(lt % tilesN); lt /= tilesN;
-  const int tm = (int)(lt % tilesM); lt /= tilesM;
-  const int no = (int)(lt % d.No); lt /= d.No;
-  const int mo = (int)(lt % d.Mo);
-  const long long t = lt / d.Mo;
-  const int m0 = tm * TBM, n0 = tn * TBN;
-  const int Mi = d.Mi, Ni = d.Ni, Ki = d.Ki;
-  const int sAmi = (int)d.sAmi, sAki = (int)d.sAki, sBki = (int)d.sBki, sBni = (int)d.sBni;
-  const double2 *Ab = d.A + t * d.sAt + mo * d.sAmo + (long long)m0 * sAmi;
-  const double2 *Bb = d.B + t * d.sBt + no * d.sBno + (long long)n0 * sBni;
-  const bool akf = sAki == 1, bnf = sBni == 1;
-  const int KT = (Ki + BKs - 1) / BKs, KTOT = d.Ko * KT;
-  constexpr int AL = TBM * BKs / 128, BL = TBN * BKs / 128;  // copies per thread per stage
-
-  auto load = [&](int slot, int kt) {
-    const int ko = kt / KT;
-    const int kb = (kt - ko * KT) * BKs;
-    const double2 *Ak = Ab + ko * d.sAko + (long long)kb * sAki;
-    const double2 *Bk = Bb + ko * d.sBko + (long long)kb * sBki;
-    double2 *as = As + slot * Cfg::AE;
-    double2 *bs = Bs + slot * Cfg::BE;
-#pragma unroll
-    for (int j = 0; j < AL; ++j) {
-      const int e = tid + 128 * j;
-      int m, k;
-      if (akf) { k = e & (BKs - 1); m = e / BKs; } else { m = e % TBM; k = e / TBM; }
-      const bool v = (m0 + m < Mi) && (kb + k < Ki);
-      cp_async16(as + m * AP + k, v ? Ak + m * sAmi + k * sAki : d.A, v);
-    }
-#pragma unroll
-    for (int j = 0; j < BL; ++j) {
-      const int e = tid + 128 * j;
-      int n, k;
-      if (bnf) { n = e % TBN; k = e / TBN; } else { k = e & (BKs - 1); n = e / BKs; }
-      const bool v = (n0 + n < Ni) && (kb + k < Ki);
-      cp_async16(bs + k * BP + n, v ? Bk + k * sBki + n * sBni : d.B, v);
-    }
-  };
-
-  double cr[MI][NJ][2], ci[MI][NJ][2];
-#pragma unroll
-  for (int i = 0; i < MI; ++i)
-#pragma unroll
-    for (int j = 0; j < NJ; ++j) { cr[i][j][0] = cr[i][j][1] = ci[i][j][0] = ci[i][j][1] = 0.0; }
-#pragma unroll
-  for (int s = 0; s < TST - 1; ++s) {
-    if (s < KTOT) load(s, s);
-    cp_async_commit();
-  }
-  for (int kt = 0; kt < KTOT; ++kt) {
-    cp_async_wait<TST - 2>();
-    __syncthreads();
-    const int nk = kt + TST - 1;
-    if (nk < KTOT) load(nk % TST, nk);
-    cp_async_commit();
-    const double2 *as = As + (kt % TST) * Cfg::AE;
-    const double2 *bs = Bs + (kt % TST) * Cfg::BE;
-#pragma unroll
-    for (int kq = 0; kq < BKs / 4; ++kq) {
-      double ar[MI], ai[MI], br[NJ], bi[NJ];
-#pragma unroll
-      for (int i = 0; i < MI; ++i) {
-        const double2 a = as[(wm * MI * 8 + i * 8 + (lane >> 2)) * AP + kq * 4 + (lane & 3)];
-        ar[i] = a.x; ai[i] = a.y;
-      }
-#pragma unroll
-      for (int j = 0; j < NJ; ++j) {
-        const double2 b = bs[(kq * 4 + (lane & 3)) * BP + wn * NJ * 8 + j * 8 + (lane >> 2)];
-        br[j] = b.x; bi[j] = b.y;
-      }
-#pragma unroll
-      for (int i = 0; i < MI; ++i)
-#pragma unroll
-        for (int j = 0; j < NJ; ++j) {
-          dmma(cr[i][j][0], cr[i][j][1], ar[i], br[j]);
-          dmma(ci[i][j][0], ci[i][j][1], ar[i], bi[j]);
-        }
-#pragma unroll
-      for (int i = 0; i < MI; ++i)
-#pragma unroll
-        for (int j = 0; j < NJ; ++j) {
-          dmma(cr[i][j][0], cr[i][j][1], dneg(ai[i]), bi[j]);
-          dmma(ci[i][j][0], ci[i][j][1], ai[i], br[j]);
-        }
-    }
-  }
-  cp_async_wait<0>();
-  double2 *C = d.C + t * d.sCt + mo * d.sCmo + no * d.sCno;
-  const long long sCmi = d.sCmi, sCni = d.sCni;
-#pragma unroll
-  for (int i = 0; i < MI; ++i) {
-    const int m = m0 + wm * MI * 8 + i * 8 + (lane >> 2);
-    if (m >= Mi) continue;
-#pragma unroll
-    for (int j = 0; j < NJ; ++j) {
-      const int n = n0 + wn * NJ * 8 + j * 8 + (lane & 3) * 2;
-      double2 *cp = C + (long long)m * sCmi + (long long)n * sCni;
-      if (n < Ni) cp[0] = make_double2(cr[i][j][0], ci[i][j][0]);
-      if (n + 1 < Ni) cp[sCni] = make_double2(cr[i][j][1], ci[i][j][1]);
-    }
-  }
-}
-
 // ---------------------------------------------------------------- persistent GEMM (v2, 3M)
 //
 // The production GEMM.  Persistent CTAs (2 per SM) take every G-th tile and run one
@@ -674,308 +535,6 @@ __device__ __forceinline__ void zgemm_persistent_body(const GemmDesc *__restrict
   cp_async_wait<0>();
 }
 
-// ---------------------------------------------------------------- warp-specialized GEMM (v3)
-//
-// Producer/consumer split so the DMMA warps execute nothing but shared-memory fragment loads
-// and DMMAs (the v1/v2 captures show long-scoreboard stalls from the cp.async address math
-// and register reuse inside the DMMA warps):
-//  * warp 4 (producer) streams tile rows with 1-D bulk async copies
-//    (cp.async.bulk ... mbarrier::complete_tx, SASS UBLKCP) into padded shared-memory rows,
-//    zero-filling ragged rows/tails itself, and signals a "full" mbarrier per stage;
-//  * warps 0-3 (consumers) wait on "full", run the 32×32-complex DMMA warp tiles, release
-//    the stage on an "empty" mbarrier, and write C from registers at the end of each tile;
-//  * persistent CTAs over contiguous tile ranges; the pipeline runs across tile boundaries.
-// The smem orientation follows the global one (A [m][k] or [k][m], B [k][n] or [n][k]) so
-// every bulk copy is a contiguous run; the fragment loads are specialised per orientation
-// (all four are bank-conflict free with the pitches below).  Operands with no unit-stride
-// inner index use zgemm_dmma_kernel.
-
-constexpr int NCW = 4;                    // consumer warps
-constexpr int NPW = 4;                    // producer warps (outstanding cp.async spread over 128 lanes)
-constexpr int NT3 = (NCW + NPW) * 32;
-constexpr int PITCH_MK = BK2 + 4;         // [m][k] / [n][k]: 320 B rows
-constexpr int PITCH_KM = BM + 2;          // [k][m] / [k][n]: 1056 B rows
-
-template <bool A_MK, bool B_KN>
-struct V3Cfg {
-  static constexpr int A_ELEMS = A_MK ? BM * PITCH_MK : BK2 * PITCH_KM;
-  static constexpr int B_ELEMS = B_KN ? BK2 * PITCH_KM : BN * PITCH_MK;
-  static constexpr int STAGE = A_ELEMS + B_ELEMS;
-  static constexpr int ST = (220 * 1024) / (STAGE * 16) > 6 ? 6 : (220 * 1024) / (STAGE * 16);
-  static constexpr int SMEM = ST * STAGE * 16 + 2 * ST * 8;
-};
-
-__device__ __forceinline__ uint32_t smem_u32(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
-
-__device__ __forceinline__ void mbar_init(uint32_t bar, uint32_t count) {
-  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;\n" ::"r"(bar), "r"(count));
-}
-__device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
-  uint32_t done;
-  do {
-    asm volatile(
-        "{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n selp.u32 %0, 1, 0, p;\n}\n"
-        : "=r"(done)
-        : "r"(bar), "r"(parity)
-        : "memory");
-  } while (!done);
-}
-__device__ __forceinline__ void mbar_arrive(uint32_t bar) {
-  asm volatile("{\n .reg .b64 st;\n mbarrier.arrive.shared::cta.b64 st, [%0];\n}\n" ::"r"(bar) : "memory");
-}
-__device__ __forceinline__ void mbar_arrive_tx(uint32_t bar, uint32_t bytes) {
-  asm volatile("{\n .reg .b64 st;\n mbarrier.arrive.expect_tx.shared::cta.b64 st, [%0], %1;\n}\n" ::"r"(bar),
-               "r"(bytes)
-               : "memory");
-}
-__device__ __forceinline__ void bulk_g2s(uint32_t dst, const void *src, uint32_t bytes, uint32_t bar) {
-  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];\n" ::"r"(dst),
-               "l"(src), "r"(bytes), "r"(bar)
-               : "memory");
-}
-
-struct V3Tile {  // what both roles need about one tile
-  const GemmDesc *d;
-  long long t;
-  int mo, no, m0, n0, KT, KTOT;
-};
-
-__device__ __forceinline__ void v3_decode(const GemmDesc *__restrict__ descs, int n_desc, int &task, long long tile,
-                                          V3Tile &T) {
-  while (task + 1 < n_desc && descs[task + 1].tile_begin <= tile) ++task;
-  const GemmDesc *d = descs + task;
-  long long lt = tile - d->tile_begin;
-  const int tilesN = d->tilesN, tilesM = d->tilesM, No = d->No, Mo = d->Mo;
-  const int tn = (int)(lt % tilesN); lt /= tilesN;
-  const int tm = (int)(lt % tilesM); lt /= tilesM;
-  T.no = (int)(lt % No); lt /= No;
-  T.mo = (int)(lt % Mo);
-  T.t = lt / Mo;
-  T.m0 = tm * BM;
-  T.n0 = tn * BN;
-  T.d = d;
-  T.KT = (d->Ki + BK2 - 1) / BK2;
-  T.KTOT = d->Ko * T.KT;
-}
-
-template <bool A_MK, bool B_KN>
-__device__ __forceinline__ void zgemm_dmma_ws_body(const GemmDesc *__restrict__ descs, int n_desc, long long total) {
-  using Cfg = V3Cfg<A_MK, B_KN>;
-  constexpr int ST3 = Cfg::ST;
-  extern __shared__ __align__(128) double2 smem[];
-  uint64_t *bars = reinterpret_cast<uint64_t *>(smem + ST3 * Cfg::STAGE);  // full[ST3], empty[ST3]
-  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-
-  const long long per = total / gridDim.x, rem = total % gridDim.x;
-  const long long t_begin = blockIdx.x * per + min((long long)blockIdx.x, rem);
-  const long long t_end = t_begin + per + ((long long)blockIdx.x < rem ? 1 : 0);
-  if (t_begin >= t_end) return;
-  int task = 0;
-  {
-    int lo = 0, hi = n_desc - 1;
-    while (lo < hi) {
-      int mid = (lo + hi + 1) >> 1;
-      if (descs[mid].tile_begin <= t_begin) lo = mid; else hi = mid - 1;
-    }
-    task = lo;
-  }
-  if (tid == 0) {
-    for (int s = 0; s < ST3; ++s) {
-      mbar_init(smem_u32(&bars[s]), 32 * NPW);
-      mbar_init(smem_u32(&bars[ST3 + s]), NCW);
-    }
-    asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
-  }
-  __syncthreads();
-
-  if (warp < NPW) {
-    // ------------------------------------------------------------ producer warps
-    // Warp 0 on purpose: the SMSP arbiter favours the highest warp id, so the DMMA warp that
-    // shares this SMSP (warp 4) wins every issue slot it can use and the producer fills the
-    // cycles between its DMMAs (with the producer as warp 4 the CTA ran at the pace of the
-    // starved consumer: 65% DMMA-pipe activity, profiles/ncu_gemm_r01_v4.json).
-    // Per-thread 16-byte cp.async (LDGSTS) along the unit-stride index of each operand (the
-    // bulk-copy variant serialised one UBLKCP per row through the uniform datapath and could
-    // not keep up), zero-fill by src-size 0 for ragged rows/tails, and completion signalled
-    // to the stage's "full" mbarrier by cp.async.mbarrier.arrive.noinc from every lane.
-    int step = 0;
-    for (long long tile = t_begin; tile < t_end; ++tile) {
-      V3Tile T;
-      v3_decode(descs, n_desc, task, tile, T);
-      const GemmDesc &d = *T.d;
-      const int Ki = d.Ki;
-      const long long sAmi = d.sAmi, sAki = d.sAki, sBki = d.sBki, sBni = d.sBni;
-      const double2 *Ab = d.A + T.t * d.sAt + T.mo * d.sAmo + (long long)T.m0 * sAmi;
-      const double2 *Bb = d.B + T.t * d.sBt + T.no * d.sBno + (long long)T.n0 * sBni;
-      const int mv = min(BM, d.Mi - T.m0), nv = min(BN, d.Ni - T.n0);  // valid rows / cols
-      for (int kt = 0; kt < T.KTOT; ++kt, ++step) {
-        const int slot = step % ST3;
-        const uint32_t full = smem_u32(&bars[slot]), empty = smem_u32(&bars[ST3 + slot]);
-        mbar_wait(empty, ((step / ST3) & 1) ^ 1);
-        const int ko = kt / T.KT;
-        const int kb = (kt - ko * T.KT) * BK2;
-        const int kv = min(BK2, Ki - kb);  // valid k in this step
-        const double2 *Ak = Ab + ko * d.sAko + (long long)kb * sAki;
-        const double2 *Bk = Bb + ko * d.sBko + (long long)kb * sBki;
-        double2 *as = smem + slot * Cfg::STAGE;
-        double2 *bs = as + Cfg::A_ELEMS;
-#pragma unroll 4
-        for (int j = 0; j < (BM * BK2) / (32 * NPW); ++j) {
-          const int e = tid + 32 * NPW * j;
-          int m, k;
-          if (A_MK) { k = e & (BK2 - 1); m = e / BK2; } else { m = e & (BM - 1); k = e / BM; }
-          const bool v = m < mv && k < kv;
-          const double2 *src = v ? Ak + m * sAmi + k * sAki : d.A;
-          cp_async16(A_MK ? as + m * PITCH_MK + k : as + k * PITCH_KM + m, src, v);
-        }
-#pragma unroll 4
-        for (int j = 0; j < (BN * BK2) / (32 * NPW); ++j) {
-          const int e = tid + 32 * NPW * j;
-          int n, k;
-          if (B_KN) { n = e & (BN - 1); k = e / BN; } else { k = e & (BK2 - 1); n = e / BK2; }
-          const bool v = n < nv && k < kv;
-          const double2 *src = v ? Bk + k * sBki + n * sBni : d.B;
-          cp_async16(B_KN ? bs + k * PITCH_KM + n : bs + n * PITCH_MK + k, src, v);
-        }
-        asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];\n" ::"r"(full) : "memory");
-      }
-    }
-    asm volatile("cp.async.wait_all;\n" ::: "memory");
-    return;
-  }
-
-  // -------------------------------------------------------------- consumer warps
-  // One consumer warp per SMSP: it must issue a DMMA every 16 cycles, so its shared-memory
-  // fragment loads for k-quad q+1 are issued before the DMMAs of q (double-buffered
-  // fragments), and the next stage is awaited one k-quad early.
-  const int cw = warp - NPW;  // consumer index 0..3
-  const int wm = cw >> 1, wn = cw & 1;
-  double cr[4][4][2], ci[4][4][2];
-#pragma unroll
-  for (int i = 0; i < 4; ++i)
-#pragma unroll
-    for (int j = 0; j < 4; ++j) { cr[i][j][0] = cr[i][j][1] = ci[i][j][0] = ci[i][j][1] = 0.0; }
-  double fa[2][4][2], fb[2][4][2];  // [buffer][i or j][re, im]
-  auto load_frags = [&](int buf, const double2 *as, const double2 *bs, int kq) {
-#pragma unroll
-    for (int i = 0; i < 4; ++i) {
-      const int m = wm * 32 + i * 8 + (lane >> 2), k = kq * 4 + (lane & 3);
-      const double2 a = A_MK ? as[m * PITCH_MK + k] : as[k * PITCH_KM + m];
-      fa[buf][i][0] = a.x; fa[buf][i][1] = a.y;
-    }
-#pragma unroll
-    for (int j = 0; j < 4; ++j) {
-      const int n = wn * 32 + j * 8 + (lane >> 2), k = kq * 4 + (lane & 3);
-      const double2 b = B_KN ? bs[k * PITCH_KM + n] : bs[n * PITCH_MK + k];
-      fb[buf][j][0] = b.x; fb[buf][j][1] = b.y;
-    }
-  };
-  auto mma_quad = [&](int buf) {
-#pragma unroll
-    for (int i = 0; i < 4; ++i)
-#pragma unroll
-      for (int j = 0; j < 4; ++j) {
-        dmma(cr[i][j][0], cr[i][j][1], fa[buf][i][0], fb[buf][j][0]);
-        dmma(ci[i][j][0], ci[i][j][1], fa[buf][i][0], fb[buf][j][1]);
-      }
-#pragma unroll
-    for (int i = 0; i < 4; ++i)
-#pragma unroll
-      for (int j = 0; j < 4; ++j) {
-        dmma(cr[i][j][0], cr[i][j][1], dneg(fa[buf][i][1]), fb[buf][j][1]);
-        dmma(ci[i][j][0], ci[i][j][1], fa[buf][i][1], fb[buf][j][0]);
-      }
-  };
-  // the whole CTA range is one sequence of k-steps; count them
-  int step = 0;
-  V3Tile T;
-  long long tile = t_begin;
-  v3_decode(descs, n_desc, task, tile, T);
-  int kt = 0;
-  mbar_wait(smem_u32(&bars[0]), 0);
-  load_frags(0, smem, smem + Cfg::A_ELEMS, 0);
-  for (;;) {
-    const int slot = step % ST3;
-    const double2 *as = smem + slot * Cfg::STAGE;
-    const double2 *bs = as + Cfg::A_ELEMS;
-    // is there a next k-step (this tile or the next)?
-    const bool last_k = (kt + 1 == T.KTOT);
-    const bool has_next = !last_k || (tile + 1 < t_end);
-    const int nslot = (slot + 1 == ST3) ? 0 : slot + 1;
-    const double2 *nas = smem + nslot * Cfg::STAGE;
-#pragma unroll
-    for (int kq = 0; kq < BK2 / 4; ++kq) {
-      const int cur = kq & 1;
-      if (kq + 1 < BK2 / 4) {
-        load_frags(cur ^ 1, as, bs, kq + 1);
-      } else if (has_next) {
-        mbar_wait(smem_u32(&bars[nslot]), ((step + 1) / ST3) & 1);
-        load_frags(cur ^ 1, nas, nas + Cfg::A_ELEMS, 0);
-      }
-      if (kq + 1 == BK2 / 4) {  // every fragment of this stage is in registers: release it
-        __syncwarp();
-        if (lane == 0) mbar_arrive(smem_u32(&bars[ST3 + slot]));
-      }
-      mma_quad(cur);
-    }
-    ++step;
-    if (!last_k) { ++kt; continue; }
-    // tile done: epilogue from registers (the producer keeps filling the next stages)
-    if (T.d->D) {  // fused final contraction: partial Σ C·D of this warp's 32×32 block
-      const GemmDesc &d = *T.d;
-      const double2 *Dp = d.D + T.t * d.sDt + T.mo * d.sDmo + T.no * d.sDno;
-      const long long sDmi = d.sDmi, sDni = d.sDni;
-      const int Mi = d.Mi, Ni = d.Ni;
-      double pr = 0.0, pim = 0.0;
-#pragma unroll
-      for (int i = 0; i < 4; ++i) {
-        const int m = T.m0 + wm * 32 + i * 8 + (lane >> 2);
-#pragma unroll
-        for (int j = 0; j < 4; ++j) {
-          const int n = T.n0 + wn * 32 + j * 8 + (lane & 3) * 2;
-#pragma unroll
-          for (int h = 0; h < 2; ++h) {
-            if (m < Mi && n + h < Ni) {
-              const double2 y = Dp[(long long)m * sDmi + (long long)(n + h) * sDni];
-              pr += cr[i][j][h] * y.x - ci[i][j][h] * y.y;
-              pim += cr[i][j][h] * y.y + ci[i][j][h] * y.x;
-            }
-          }
-          cr[i][j][0] = cr[i][j][1] = ci[i][j][0] = ci[i][j][1] = 0.0;
-        }
-      }
-#pragma unroll
-      for (int off = 16; off > 0; off >>= 1) {
-        pr += __shfl_xor_sync(0xffffffffu, pr, off);
-        pim += __shfl_xor_sync(0xffffffffu, pim, off);
-      }
-      if (lane == 0) d.part[(tile - d.tile_begin) * NCW + cw] = make_double2(pr, pim);
-    } else {
-      const GemmDesc &d = *T.d;
-      double2 *C = d.C + T.t * d.sCt + T.mo * d.sCmo + T.no * d.sCno;
-      const long long sCmi = d.sCmi, sCni = d.sCni;
-      const int Mi = d.Mi, Ni = d.Ni;
-#pragma unroll
-      for (int i = 0; i < 4; ++i) {
-        const int m = T.m0 + wm * 32 + i * 8 + (lane >> 2);
-#pragma unroll
-        for (int j = 0; j < 4; ++j) {
-          const int n = T.n0 + wn * 32 + j * 8 + (lane & 3) * 2;
-          if (m < Mi) {
-            double2 *cp = C + (long long)m * sCmi + (long long)n * sCni;
-            if (n < Ni) cp[0] = make_double2(cr[i][j][0], ci[i][j][0]);
-            if (n + 1 < Ni) cp[sCni] = make_double2(cr[i][j][1], ci[i][j][1]);
-          }
-          cr[i][j][0] = cr[i][j][1] = ci[i][j][0] = ci[i][j][1] = 0.0;
-        }
-      }
-    }
-    if (++tile >= t_end) break;
-    v3_decode(descs, n_desc, task, tile, T);
-    kt = 0;
-  }
-}
-
 // ---------------------------------------------------------------- dot / trace
 
 constexpr int DT = 256;
@@ -1121,66 +680,40 @@ __global__ void accumulate_kernel(double2 *dst, const double2 *src, long long n)
 __global__ void __launch_bounds__(NT, 2) zgemm_dmma_kernel(const __grid_constant__ GemmBatch b, long long total) {
   zgemm_dmma_kernel_body(b.d, b.n, total);
 }
-template <int TBM, int TBN, int TST, int MINB>
-__global__ void __launch_bounds__(128, MINB) zgemm_small(const __grid_constant__ GemmBatch b, long long total) {
-  zgemm_small_body<TBM, TBN, TST>(b.d, b.n, total);
-}
 template <int NWM, int NWN, int WTM, int WTN, bool M3>
 __global__ void __launch_bounds__(NWM * NWN * 32, 2)
     zgemm_persistent(const __grid_constant__ GemmBatch b, long long total) {
   zgemm_persistent_body<NWM, NWN, WTM, WTN, M3>(b.d, b.n, total);
 }
-template <int NWM, int NWN, int WTM, int WTN, bool M3>
-__global__ void __launch_bounds__(NWM * NWN * 32, 1)
-    zgemm_persistent1(const __grid_constant__ GemmBatch b, long long total) {
-  zgemm_persistent_body<NWM, NWN, WTM, WTN, M3>(b.d, b.n, total);
-}
-template <bool A_MK, bool B_KN>
-__global__ void __launch_bounds__(NT3, 1) zgemm_dmma_ws(const __grid_constant__ GemmBatch b, long long total) {
-  zgemm_dmma_ws_body<A_MK, B_KN>(b.d, b.n, total);
-}
-__global__ void __launch_bounds__(DT) zdot_kernel(const __grid_constant__ DotBatch b) { zdot_body(b.d, b.n); }
 
-template <bool A_MK, bool B_KN>
-cudaError_t launch_ws(const GemmBatch *b, long long total, int sms, cudaStream_t st) {
-  using Cfg = V3Cfg<A_MK, B_KN>;
-  static bool attr = false;
-  if (!attr) {
-    cudaError_t e = cudaFuncSetAttribute(zgemm_dmma_ws<A_MK, B_KN>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         Cfg::SMEM);
-    if (e != cudaSuccess) return e;
-    attr = true;
-  }
-  long long grid = sms;  // one CTA (4 DMMA warps + 1 producer) per SM
-  if (grid > total) grid = total;
-  zgemm_dmma_ws<A_MK, B_KN><<<(unsigned)grid, NT3, Cfg::SMEM, st>>>(*b, total);
-  return cudaGetLastError();
-}
+__global__ void __launch_bounds__(DT) zdot_kernel(const __grid_constant__ DotBatch b) { zdot_body(b.d, b.n); }
 
 }  // namespace
 
 int gemm_variant() {
-  // MICCO_GEMM = 1 per-tile 64×64, 2 persistent 64×64 4M, 3 warp-specialized, 5 persistent 64×32 3M
-  // (default: 19.7k vs 18.8k graphs/s for 2 on the bench workload, profiles/bench_r01_v4.json),
-  // 6 small 32×32 (4 stages, 3 CTAs/SM), 7 64×32, 8 32×32 (3 stages, 4 CTAs/SM)
+  // MICCO_GEMM = 5 (default) persistent 64×32 tiles, 3M complex products;
+  //              2 persistent 64×64 tiles, 4M;  1 per-tile 64×64 4M (also the gather kernel).
+  // Measured on the bench workload: 5 → 19.9k, 2 → 18.9k graphs/s (profiles/bench_r01_v6.json).
+  // Earlier experiments (warp-specialised producer/consumer, small 32×32 tiles, 8-warp 3M)
+  // are in DESIGN.md §6's history table; all were slower and were removed.
   static int variant = -1;
   if (variant < 0) {
     const char *e = getenv("MICCO_GEMM");
-    variant = (e && e[0] >= '1' && e[0] <= '8') ? e[0] - '0' : 5;
+    variant = (e && (e[0] == '1' || e[0] == '2' || e[0] == '5')) ? e[0] - '0' : 5;
   }
   return variant;
 }
 
 void gemm_tile_shape(int cls, int *bm, int *bn) {
-  const int v = gemm_variant();
   *bm = 64;
   *bn = 64;
   if (cls == 4) return;  // gather kernel (v1)
-  if (v == 6 || v == 8) { *bm = 32; *bn = 32; }
-  if (v == 7 || v == 5) { *bm = 64; *bn = 32; }
+  if (gemm_variant() == 5) *bn = 32;
 }
 
-bool gemm_uses_3m(int cls) { return cls != 4 && (gemm_variant() == 5 || gemm_variant() == 4); }
+bool gemm_uses_3m(int cls) { return cls != 4 && gemm_variant() == 5; }
+
+bool gemm_fused_dot_ok() { return gemm_variant() != 1; }
 
 cudaError_t launch_gemm_group(const GemmBatch *b, long long total_tiles, int cls, cudaStream_t st) {
   static bool attr_set = false;  // per process; the attribute is per-function, all devices
@@ -1200,59 +733,18 @@ cudaError_t launch_gemm_group(const GemmBatch *b, long long total_tiles, int cls
   int dev = 0, sms = 148;
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-  if (variant == 1 || cls == 4) {
+  if (variant == 1 || cls == 4) {  // per-tile kernel; the only one that gathers strided operands
     long long grid = total_tiles < (1LL << 30) ? total_tiles : (1LL << 30);
     zgemm_dmma_kernel<<<(unsigned)grid, NT, GEMM_SMEM, st>>>(*b, total_tiles);
     return cudaGetLastError();
   }
-  if (variant == 6 || variant == 7 || variant == 8) {
-    // tile sizes must match the host's tilesM/tilesN (kGemmBM/BN for the other variants)
-    long long grid = total_tiles;
-    if (variant == 6) {
-      using C6 = SmallCfg<32, 32, 4>;
-      static bool a6 = false;
-      if (!a6) { cudaFuncSetAttribute(zgemm_small<32, 32, 4, 3>, cudaFuncAttributeMaxDynamicSharedMemorySize, C6::SMEM); a6 = true; }
-      zgemm_small<32, 32, 4, 3><<<(unsigned)grid, 128, C6::SMEM, st>>>(*b, total_tiles);
-    } else if (variant == 7) {
-      using C7 = SmallCfg<64, 32, 4>;
-      static bool a7 = false;
-      if (!a7) { cudaFuncSetAttribute(zgemm_small<64, 32, 4, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, C7::SMEM); a7 = true; }
-      zgemm_small<64, 32, 4, 2><<<(unsigned)grid, 128, C7::SMEM, st>>>(*b, total_tiles);
-    } else {
-      using C8 = SmallCfg<32, 32, 3>;
-      static bool a8 = false;
-      if (!a8) { cudaFuncSetAttribute(zgemm_small<32, 32, 3, 4>, cudaFuncAttributeMaxDynamicSharedMemorySize, C8::SMEM); a8 = true; }
-      zgemm_small<32, 32, 3, 4><<<(unsigned)grid, 128, C8::SMEM, st>>>(*b, total_tiles);
-    }
-    return cudaGetLastError();
-  }
-  if (variant == 4) {  // 3M, 8 warps of 32×16 on a 64×64 tile, one CTA per SM (255 registers)
-    static bool a4 = false;
-    if (!a4) {
-      cudaFuncSetAttribute(zgemm_persistent1<2, 4, 32, 16, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                           PCfg<64, 64>::SMEM);
-      a4 = true;
-    }
-    long long grid = sms;
-    if (grid > total_tiles) grid = total_tiles;
-    zgemm_persistent1<2, 4, 32, 16, true><<<(unsigned)grid, 256, PCfg<64, 64>::SMEM, st>>>(*b, total_tiles);
-    return cudaGetLastError();
-  }
-  if (variant == 2 || variant == 5) {
-    long long grid = 2LL * sms;  // 2 resident CTAs per SM (112 KB smem each)
-    if (grid > total_tiles) grid = total_tiles;
-    if (variant == 2)
-      zgemm_persistent<2, 2, 32, 32, false><<<(unsigned)grid, 128, PCfg<64, 64>::SMEM, st>>>(*b, total_tiles);
-    else  // 5: 3M complex products, 64×32 CTA tile
-      zgemm_persistent<2, 2, 32, 16, true><<<(unsigned)grid, 128, PCfg<64, 32>::SMEM, st>>>(*b, total_tiles);
-    return cudaGetLastError();
-  }
-  switch (cls) {
-    case 0: return launch_ws<true, true>(b, total_tiles, sms, st);
-    case 1: return launch_ws<true, false>(b, total_tiles, sms, st);
-    case 2: return launch_ws<false, true>(b, total_tiles, sms, st);
-    default: return launch_ws<false, false>(b, total_tiles, sms, st);
-  }
+  long long grid = 2LL * sms;  // 2 resident CTAs per SM
+  if (grid > total_tiles) grid = total_tiles;
+  if (variant == 2)
+    zgemm_persistent<2, 2, 32, 32, false><<<(unsigned)grid, 128, PCfg<64, 64>::SMEM, st>>>(*b, total_tiles);
+  else
+    zgemm_persistent<2, 2, 32, 16, true><<<(unsigned)grid, 128, PCfg<64, 32>::SMEM, st>>>(*b, total_tiles);
+  return cudaGetLastError();
 }
 
 cudaError_t launch_dot_group(const DotBatch *b, long long total_ctas, cudaStream_t st) {

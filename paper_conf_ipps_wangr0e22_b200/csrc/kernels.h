@@ -79,6 +79,7 @@ constexpr int kGemmClasses = 5;
 int gemm_variant();
 void gemm_tile_shape(int cls, int *bm, int *bn);
 bool gemm_uses_3m(int cls);  // 3 DMMA products per complex MAC for this layout class
+bool gemm_fused_dot_ok();    // the selected persistent GEMM has the fused-dot epilogue (4 warps/CTA)
 
 // Grouped launches: descs in device memory (all of one layout class); grid covers the tiles.
 cudaError_t launch_gemm_group(const GemmBatch *b, long long total_tiles, int cls, cudaStream_t st);
