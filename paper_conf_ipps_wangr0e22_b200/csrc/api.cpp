@@ -114,13 +114,13 @@ void check_shape(int32_t rank, int32_t N) {
   if (N < 1 || N > 65536) fail(MICCO_ERR_ARG, "N out of range");
 }
 
-int32_t new_node(Context &c, int32_t rank, int32_t N) {
+int32_t new_node(Context &c, int32_t rank, int32_t N, bool allocate = true) {
   NodeRec nd;
   nd.rank = rank;
   nd.N = N;
   nd.slice_elems = 1;
   for (int i = 0; i < rank; ++i) nd.slice_elems *= N;
-  nd.host = c.arena.alloc(nd.slice_elems * (int64_t)c.Lt * 16);
+  if (allocate) nd.host = c.arena.alloc(nd.slice_elems * (int64_t)c.Lt * 16);
   c.nodes.push_back(nd);
   int32_t id = (int32_t)c.nodes.size() - 1;
   c.nodes[id].tensor = add_node_tensor(c, id);
@@ -201,37 +201,65 @@ MICCO_API micco_status micco_add_hadron_nodes_synth(micco_ctx *ctx, int32_t coun
     if (mode != MICCO_SYNTH_UNIFORM && mode != MICCO_SYNTH_INT3) fail(MICCO_ERR_ARG, "bad synth mode");
     check_shape(rank, N);
     check_lt(c, Lt);
-    std::vector<std::pair<int32_t, uint64_t>> todo;  // (node, key) to generate
+    const bool lazy = c.opt.dist_world > 0;  // multi-process: generate on first use by this rank
+    std::vector<int32_t> todo;
     for (int32_t i = 0; i < count; ++i) {
       SynthKey k{seed, keys[i], mode, rank, N, scale};
       auto it = c.node_by_synth.find(k);
       if (it != c.node_by_synth.end()) { node_ids[i] = it->second; continue; }
-      int32_t id = new_node(c, rank, N);
+      int32_t id = new_node(c, rank, N, /*allocate=*/false);
+      NodeRec &nd = c.nodes[id];
+      nd.synth = true;
+      nd.syn_seed = seed;
+      nd.syn_key = keys[i];
+      nd.syn_mode = mode;
+      nd.syn_scale = scale;
       c.node_by_synth.emplace(k, id);
-      todo.push_back({id, keys[i]});
+      todo.push_back(id);
       node_ids[i] = id;
     }
-    if (todo.empty()) return;
-    const int64_t per = c.nodes[todo[0].first].slice_elems * (int64_t)Lt;
-    // split every node into blocks so all host threads stay busy
-    const int64_t blk = 1 << 18;
-    const int64_t blocks_per = (per + blk - 1) / blk;
-    const int64_t total = blocks_per * (int64_t)todo.size();
-    unsigned nt = std::max(1u, std::min(64u, std::thread::hardware_concurrency()));
-    std::vector<std::thread> th;
-    std::atomic<int64_t> next{0};
-    for (unsigned w = 0; w < nt; ++w)
-      th.emplace_back([&] {
-        for (int64_t i; (i = next.fetch_add(1)) < total;) {
-          const auto &td = todo[i / blocks_per];
-          int64_t first = (i % blocks_per) * blk;
-          int64_t cnt = std::min(blk, per - first);
-          micco_synth_fill(c.nodes[td.first].host + 2 * first, seed, td.second, first, cnt, mode, scale);
-        }
-      });
-    for (auto &t : th) t.join();
+    if (!lazy) materialize_nodes(c, todo);
   });
 }
+
+}  // extern "C"
+
+namespace micco {
+
+void materialize_nodes(Context &c, const std::vector<int32_t> &node_ids) {
+  std::vector<int32_t> todo;
+  for (int32_t id : node_ids)
+    if (c.nodes[id].synth && !c.nodes[id].host) todo.push_back(id);
+  if (todo.empty()) return;
+  for (int32_t id : todo) c.nodes[id].host = c.arena.alloc(c.nodes[id].slice_elems * (int64_t)c.Lt * 16);
+  // split every node into blocks so all host threads stay busy
+  const int64_t blk = 1 << 18;
+  std::vector<int64_t> first_block(todo.size() + 1, 0);
+  for (size_t i = 0; i < todo.size(); ++i) {
+    const int64_t per = c.nodes[todo[i]].slice_elems * (int64_t)c.Lt;
+    first_block[i + 1] = first_block[i] + (per + blk - 1) / blk;
+  }
+  const int64_t total = first_block.back();
+  unsigned nt = std::max(1u, std::min(64u, std::thread::hardware_concurrency()));
+  std::vector<std::thread> th;
+  std::atomic<int64_t> next{0};
+  for (unsigned w = 0; w < nt; ++w)
+    th.emplace_back([&] {
+      for (int64_t b; (b = next.fetch_add(1)) < total;) {
+        const size_t i = std::upper_bound(first_block.begin(), first_block.end(), b) - first_block.begin() - 1;
+        const NodeRec &nd = c.nodes[todo[i]];
+        const int64_t per = nd.slice_elems * (int64_t)c.Lt;
+        const int64_t first = (b - first_block[i]) * blk;
+        const int64_t cnt = std::min(blk, per - first);
+        micco_synth_fill(nd.host + 2 * first, nd.syn_seed, nd.syn_key, first, cnt, nd.syn_mode, nd.syn_scale);
+      }
+    });
+  for (auto &t : th) t.join();
+}
+
+}  // namespace micco
+
+extern "C" {
 
 MICCO_API micco_status micco_add_graph(micco_ctx *ctx, int32_t n_inst, const int64_t *node_ids, int32_t n_edges,
                                        const micco_edge *edges, const int32_t *order, double coef_re,

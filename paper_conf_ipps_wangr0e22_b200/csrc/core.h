@@ -32,6 +32,13 @@ struct NodeRec {
   double *host = nullptr;   // 2 * Lt * slice_elems doubles, interleaved, t slowest
   uint64_t hash = 0;
   int32_t tensor = -1;
+  // generator descriptor of a synthetic node; in multi-process mode its data is generated on
+  // first use by this rank (host == nullptr until then), so a rank never holds nodes it
+  // does not upload
+  bool synth = false;
+  uint64_t syn_seed = 0, syn_key = 0;
+  int32_t syn_mode = 0;
+  double syn_scale = 0;
 };
 
 enum TaskKind : int8_t { TASK_GEMM = 0, TASK_DOT = 1, TASK_TRACE = 2 };
@@ -151,6 +158,10 @@ struct Context {
   Context();
   ~Context();
 };
+
+// api.cpp: generate (in parallel, into pinned memory) the data of synthetic nodes not yet
+// materialised
+void materialize_nodes(Context &ctx, const std::vector<int32_t> &node_ids);
 
 // builder.cpp
 int32_t add_node_tensor(Context &ctx, int32_t node);

@@ -329,7 +329,10 @@ struct Executor::Impl {
 
   const double *host_src(int32_t x) const {
     const TensorRec &t = c.tensors[x];
-    if (t.node >= 0) return c.nodes[t.node].host;
+    if (t.node >= 0) {
+      if (!c.nodes[t.node].host) fail(MICCO_ERR_STATE, "executor: node data not materialised");
+      return c.nodes[t.node].host;
+    }
     auto it = spill_host.find(x);
     if (it == spill_host.end()) fail(MICCO_ERR_STATE, "executor: missing host copy");
     return it->second;
@@ -643,6 +646,14 @@ struct Executor::Impl {
     }
     cached_nodes = plan.final_nodes;
     fused_dot = plan.fused_dot;
+    {  // synthetic nodes this process uploads must have host data (lazy in multi-process mode)
+      std::vector<int32_t> need;
+      for (const PlanOp &op : plan.ops)
+        if (op.kind == PlanOp::H2D && g[op.gpu].local && c.tensors[op.id].node >= 0 &&
+            !c.nodes[c.tensors[op.id].node].host)
+          need.push_back(c.tensors[op.id].node);
+      materialize_nodes(c, need);
+    }
     auto t1 = std::chrono::steady_clock::now();
 
     micco_stats st{};
