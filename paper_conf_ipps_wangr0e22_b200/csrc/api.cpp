@@ -29,6 +29,16 @@ void HostArena::release_all() {
     if (c.pinned) cudaFreeHost(c.base); else std::free(c.base);
   }
   chunks_.clear();
+  cur_ = 0;
+  for (auto &b : big_) {
+    if (b.second) cudaFreeHost(b.first); else std::free(b.first);
+  }
+  big_.clear();
+}
+
+void HostArena::rewind() {
+  for (auto &c : chunks_) c.used = 0;
+  cur_ = 0;
   for (auto &b : big_) {
     if (b.second) cudaFreeHost(b.first); else std::free(b.first);
   }
@@ -57,13 +67,14 @@ double *HostArena::alloc(int64_t bytes) {
     big_.push_back({p, pinned});
     return (double *)p;
   }
-  if (chunks_.empty() || chunks_.back().used + bytes > chunks_.back().size) {
+  while (cur_ < chunks_.size() && chunks_[cur_].used + bytes > chunks_[cur_].size) ++cur_;
+  if (cur_ == chunks_.size()) {
     bool pinned;
     char *p = raw(kChunk, pinned);
     if (!p) fail(MICCO_ERR_OOM, "host allocation failed");
     chunks_.push_back({p, kChunk, 0, pinned});
   }
-  Chunk &c = chunks_.back();
+  Chunk &c = chunks_[cur_];
   char *p = c.base + c.used;
   c.used += bytes;
   return (double *)p;

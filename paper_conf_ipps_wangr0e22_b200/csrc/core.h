@@ -119,10 +119,12 @@ class HostArena {
   double *alloc(int64_t bytes);
   bool pinned() const { return pinned_; }
   void release_all();
+  void rewind();  // forget all allocations but keep the pinned chunks for reuse
  private:
   struct Chunk { char *base; int64_t size, used; bool pinned; };
   std::vector<Chunk> chunks_;
   std::vector<std::pair<char *, bool>> big_;
+  size_t cur_ = 0;  // chunk being filled
   bool pinned_ = true;
 };
 

@@ -767,7 +767,7 @@ struct Executor::Impl {
     std::memcpy(c.corr.data(), h_corr, (size_t)c.Lt * 16);
     spill_host.clear();
     spill_ev.clear();
-    spill_arena.release_all();
+    spill_arena.rewind();  // keep the pinned spill chunks for the next execute
 
     // statistics
     for (const Timed &tm : timed) {

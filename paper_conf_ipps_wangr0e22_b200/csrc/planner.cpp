@@ -14,6 +14,7 @@
 // The output is a flat, globally ordered op list that the executor replays; in
 // multi-process mode every rank builds the identical plan.
 #include <algorithm>
+#include <climits>
 #include <cmath>
 #include <limits>
 #include <string>
@@ -154,10 +155,37 @@ Plan make_plan(const Context &ctx, const PlanInput &in) {
 
   // 1. window of every task = window of the first graph that needs it
   const int32_t W = in.window_graphs > 0 ? in.window_graphs : 256;
+  // Graphs are windowed in an order that keeps graphs sharing an intermediate together:
+  // key = the smallest id among the level-1 tasks a graph depends on (its first shared
+  // product), ties in graph order.  Shared intermediates then live for a few windows instead
+  // of the whole stream (fewer evictions and spills).  C(t) does not depend on this order
+  // (the final sum runs over graph ids in a fixed order).
+  std::vector<int32_t> gorder(G);
+  {
+    std::vector<int32_t> key(G, INT32_MAX), first1(T, -1);
+    for (int32_t t = 0; t < T; ++t) {  // smallest level-1 task reachable from each task
+      const TaskRec &tk = ctx.tasks[t];  // operands precede their consumers in id order
+      int32_t k = INT32_MAX;
+      for (int32_t op : {tk.a, tk.b}) {
+        if (op < 0) continue;
+        const int32_t pt = ctx.tensors[op].task;
+        if (pt >= 0) k = std::min(k, first1[pt]);
+      }
+      first1[t] = (k == INT32_MAX) ? t : k;
+    }
+    for (int32_t g = 0; g < G; ++g)
+      for (int32_t c = ctx.graphs[g].comp_begin; c < ctx.graphs[g].comp_end; ++c) {
+        const int32_t t0 = ctx.tensors[ctx.graph_scalars[c]].task;
+        if (t0 >= 0) key[g] = std::min(key[g], first1[t0]);
+      }
+    for (int32_t g = 0; g < G; ++g) gorder[g] = g;
+    std::stable_sort(gorder.begin(), gorder.end(), [&](int32_t x, int32_t y) { return key[x] < key[y]; });
+  }
   std::vector<int32_t> task_window(T, -1);
   std::vector<int32_t> stack;
-  for (int32_t g = 0; g < G; ++g) {
-    const int32_t w = g / W;
+  for (int32_t gi = 0; gi < G; ++gi) {
+    const int32_t g = gorder[gi];
+    const int32_t w = gi / W;
     for (int32_t c = ctx.graphs[g].comp_begin; c < ctx.graphs[g].comp_end; ++c) {
       int32_t t0 = ctx.tensors[ctx.graph_scalars[c]].task;
       if (t0 >= 0 && task_window[t0] < 0) { task_window[t0] = w; stack.push_back(t0); }
