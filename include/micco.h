@@ -214,6 +214,20 @@ MICCO_API micco_status micco_set_nccl_id(micco_ctx *ctx, const uint8_t id[128]);
 MICCO_API micco_status micco_plan(micco_ctx *ctx, int32_t n_gpus, const int32_t *reuse_bound,
                                   micco_stats *out, int32_t *assign);
 
+/* The plan itself, for host-side invariant checks: like micco_plan, then copies up to max_ops
+ * operations as 4 int32 each (kind, gpu, src, id) in replay order — kind 0 H2D (id = tensor),
+ * 1 P2P (src → gpu), 2 SPILL (D2H), 3 FREE (gpu −1 = the host spill copy), 4 COMPUTE
+ * (id = task), 5 FLUSH.  *n_ops receives the full count.  fused (optional, unique_tasks entries)
+ * receives, per task, the dot task fused into its epilogue or −1. */
+MICCO_API micco_status micco_plan_ops(micco_ctx *ctx, int32_t n_gpus, const int32_t *reuse_bound,
+                                      int64_t max_ops, int32_t *ops, int64_t *n_ops, int32_t *fused);
+
+/* The task DAG: per tensor its size in bytes (all Lt slices; 0 for per-slice scalars) and its
+ * producing task (−1 for hadron nodes); per task (kind 0 GEMM / 1 dot / 2 trace, operand a,
+ * operand b or −1, output tensor).  Arrays sized by *n_tensors / *n_tasks (query with NULL). */
+MICCO_API micco_status micco_dag(const micco_ctx *ctx, int64_t *n_tensors, int64_t *n_tasks,
+                                 int64_t *tensor_bytes, int32_t *tensor_task, int32_t *task_info);
+
 /* The scheduler alone (Alg. 1 + Alg. 2) over a stream of vectors of tensor
  * pairs, with no eviction: pairs[7*i .. 7*i+6] = (tensor1, tensor2, out, flops, bytes1,
  * bytes2, bytes_out); vec_off[v] .. vec_off[v+1] are the pairs of vector v; resident holds

@@ -300,23 +300,65 @@ MICCO_API micco_status micco_execute(micco_ctx *ctx, int32_t n_gpus, const int32
   });
 }
 
+namespace {
+Plan host_plan(Context &c, int32_t n_gpus, const int32_t *reuse_bound) {
+  if (n_gpus < 1 || n_gpus > 64) fail(MICCO_ERR_ARG, "n_gpus must be in [1, 64]");
+  if (c.opt.mem_budget_bytes <= 0) fail(MICCO_ERR_ARG, "micco_plan needs options.mem_budget_bytes");
+  PlanInput in;
+  in.n_gpus = n_gpus;
+  in.policy = c.opt.policy;
+  for (int i = 0; i < 3; ++i) in.reuse_bound[i] = reuse_bound ? reuse_bound[i] : 0;
+  in.budget.assign(n_gpus, c.opt.mem_budget_bytes);
+  in.window_graphs = c.opt.window_graphs;
+  in.keep_inputs = c.opt.keep_inputs_resident != 0;
+  in.peer_gbs = 700;
+  in.host_gbs = 55;
+  in.flops_per_s = 30e12;
+  return reuse_bound ? make_plan(c, in) : make_plan_auto(c, in);
+}
+}  // namespace
+
+MICCO_API micco_status micco_plan_ops(micco_ctx *ctx, int32_t n_gpus, const int32_t *reuse_bound, int64_t max_ops,
+                                      int32_t *ops, int64_t *n_ops, int32_t *fused) {
+  return guard(ctx, [&] {
+    Plan p = host_plan(ctx->c, n_gpus, reuse_bound);
+    if (n_ops) *n_ops = (int64_t)p.ops.size();
+    if (ops)
+      for (int64_t i = 0; i < std::min<int64_t>(max_ops, (int64_t)p.ops.size()); ++i) {
+        ops[4 * i] = p.ops[i].kind;
+        ops[4 * i + 1] = p.ops[i].gpu;
+        ops[4 * i + 2] = p.ops[i].src;
+        ops[4 * i + 3] = p.ops[i].id;
+      }
+    if (fused) std::copy(p.fused_dot.begin(), p.fused_dot.end(), fused);
+  });
+}
+
+MICCO_API micco_status micco_dag(const micco_ctx *ctx, int64_t *n_tensors, int64_t *n_tasks, int64_t *tensor_bytes,
+                                 int32_t *tensor_task, int32_t *task_info) {
+  if (!ctx) return MICCO_ERR_ARG;
+  const Context &c = ctx->c;
+  if (n_tensors) *n_tensors = (int64_t)c.tensors.size();
+  if (n_tasks) *n_tasks = (int64_t)c.tasks.size();
+  for (size_t x = 0; x < c.tensors.size(); ++x) {
+    if (tensor_bytes) tensor_bytes[x] = c.tensors[x].rank > 0 ? c.tensors[x].bytes(c.Lt) : 0;
+    if (tensor_task) tensor_task[x] = c.tensors[x].task;
+  }
+  if (task_info)
+    for (size_t t = 0; t < c.tasks.size(); ++t) {
+      task_info[4 * t] = c.tasks[t].kind;
+      task_info[4 * t + 1] = c.tasks[t].a;
+      task_info[4 * t + 2] = c.tasks[t].b;
+      task_info[4 * t + 3] = c.tasks[t].out;
+    }
+  return MICCO_OK;
+}
+
 MICCO_API micco_status micco_plan(micco_ctx *ctx, int32_t n_gpus, const int32_t *reuse_bound, micco_stats *out,
                                   int32_t *assign) {
   return guard(ctx, [&] {
     Context &c = ctx->c;
-    if (n_gpus < 1 || n_gpus > 64) fail(MICCO_ERR_ARG, "n_gpus must be in [1, 64]");
-    if (c.opt.mem_budget_bytes <= 0) fail(MICCO_ERR_ARG, "micco_plan needs options.mem_budget_bytes");
-    PlanInput in;
-    in.n_gpus = n_gpus;
-    in.policy = c.opt.policy;
-    for (int i = 0; i < 3; ++i) in.reuse_bound[i] = reuse_bound ? reuse_bound[i] : 0;
-    in.budget.assign(n_gpus, c.opt.mem_budget_bytes);
-    in.window_graphs = c.opt.window_graphs;
-    in.keep_inputs = c.opt.keep_inputs_resident != 0;
-    in.peer_gbs = 700;
-    in.host_gbs = 55;
-    in.flops_per_s = 30e12;
-    Plan p = reuse_bound ? make_plan(c, in) : make_plan_auto(c, in);
+    Plan p = host_plan(c, n_gpus, reuse_bound);
     if (out) {
       micco_stats s{};
       s.struct_size = sizeof(s);

@@ -68,7 +68,8 @@ class micco_stats(ctypes.Structure):
 EXPORTS = ["micco_options_default", "micco_create", "micco_destroy", "micco_add_hadron_node",
            "micco_add_hadron_nodes_synth", "micco_add_graph", "micco_execute", "micco_get_correlator",
            "micco_get_graph_value", "micco_last_error", "micco_get_stats", "micco_release_cache",
-           "micco_nccl_unique_id", "micco_set_nccl_id", "micco_plan", "micco_debug_schedule"]
+           "micco_nccl_unique_id", "micco_set_nccl_id", "micco_plan", "micco_plan_ops", "micco_dag",
+           "micco_debug_schedule"]
 
 _lib = None
 
@@ -104,13 +105,17 @@ def lib() -> ctypes.CDLL:
         L.micco_nccl_unique_id.argtypes = [P(ctypes.c_uint8)]
         L.micco_set_nccl_id.argtypes = [vp, P(ctypes.c_uint8)]
         L.micco_plan.argtypes = [vp, ctypes.c_int32, P(ctypes.c_int32), P(micco_stats), P(ctypes.c_int32)]
+        L.micco_plan_ops.argtypes = [vp, ctypes.c_int32, P(ctypes.c_int32), ctypes.c_int64, P(ctypes.c_int32),
+                                     P(ctypes.c_int64), P(ctypes.c_int32)]
+        L.micco_dag.argtypes = [vp, P(ctypes.c_int64), P(ctypes.c_int64), P(ctypes.c_int64), P(ctypes.c_int32),
+                                P(ctypes.c_int32)]
         L.micco_debug_schedule.argtypes = [ctypes.c_int32, P(ctypes.c_int32), ctypes.c_double, ctypes.c_int32,
                                            P(ctypes.c_int64), P(ctypes.c_double), ctypes.c_int32,
                                            P(ctypes.c_int64), P(ctypes.c_int32)]
         for f in ("micco_create", "micco_add_hadron_node", "micco_add_hadron_nodes_synth", "micco_add_graph",
                   "micco_execute", "micco_get_correlator", "micco_get_graph_value", "micco_get_stats",
                   "micco_release_cache", "micco_nccl_unique_id", "micco_set_nccl_id", "micco_plan",
-                  "micco_debug_schedule"):
+                  "micco_plan_ops", "micco_dag", "micco_debug_schedule"):
             getattr(L, f).restype = ctypes.c_int
         _lib = L
     return _lib
@@ -229,6 +234,32 @@ def micco_plan(ctx, n_gpus: int, reuse_bound: Optional[Sequence[int]] = None, n_
     _check(ctx, lib().micco_plan(ctx, int(n_gpus), bd, ctypes.byref(s),
                                  None if assign is None else _ptr(assign, ctypes.c_int32)))
     return s.as_dict(), (None if assign is None else assign[:n_tasks])
+
+
+def micco_plan_ops(ctx, n_gpus: int, reuse_bound: Optional[Sequence[int]] = None):
+    """(ops[n, 4] = kind, gpu, src, id in replay order; fused[task] = fused dot task or -1)."""
+    bd = None if reuse_bound is None else (ctypes.c_int32 * 3)(*[int(x) for x in reuse_bound])
+    n = ctypes.c_int64()
+    _check(ctx, lib().micco_plan_ops(ctx, int(n_gpus), bd, 0, None, ctypes.byref(n), None))
+    nt = ctypes.c_int64()
+    _check(ctx, lib().micco_dag(ctx, None, ctypes.byref(nt), None, None, None))
+    ops = np.zeros((max(1, n.value), 4), dtype=np.int32)
+    fused = np.full(max(1, nt.value), -1, dtype=np.int32)
+    _check(ctx, lib().micco_plan_ops(ctx, int(n_gpus), bd, n.value, _ptr(ops, ctypes.c_int32), ctypes.byref(n),
+                                     _ptr(fused, ctypes.c_int32)))
+    return ops[:n.value], fused[:nt.value]
+
+
+def micco_dag(ctx):
+    """(tensor_bytes[nT], tensor_task[nT], task_info[nK, 4] = kind, a, b, out)."""
+    nT, nK = ctypes.c_int64(), ctypes.c_int64()
+    _check(ctx, lib().micco_dag(ctx, ctypes.byref(nT), ctypes.byref(nK), None, None, None))
+    tb = np.zeros(max(1, nT.value), dtype=np.int64)
+    tt = np.zeros(max(1, nT.value), dtype=np.int32)
+    ti = np.zeros((max(1, nK.value), 4), dtype=np.int32)
+    _check(ctx, lib().micco_dag(ctx, None, None, _ptr(tb, ctypes.c_int64), _ptr(tt, ctypes.c_int32),
+                                _ptr(ti, ctypes.c_int32)))
+    return tb[:nT.value], tt[:nT.value], ti[:nK.value]
 
 
 def micco_nccl_unique_id() -> bytes:
