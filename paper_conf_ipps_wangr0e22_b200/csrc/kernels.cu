@@ -475,27 +475,36 @@ __device__ __forceinline__ void zgemm_persistent_body(const GemmDesc *__restrict
         // fused final contraction: this warp's partial Σ C·D (no C written)
         const GemmDesc &dd = descs[task_c];
         const long long sDmi = dd.sDmi, sDni = dd.sDni;
+        // partner loads issued CH rows at a time before their use (3M: all rows, one round
+        // trip to L2 where the block was prefetched; 4M: one row, its registers are full)
+        constexpr int CH = M3 ? MI : 1;
         double pr = 0.0, pim = 0.0;
 #pragma unroll
-        for (int i = 0; i < MI; ++i) {
-          const int m = S.m0 + wm * WTM + i * 8 + (lane >> 2);
-          double2 y[NJ][2];
+        for (int i0 = 0; i0 < MI; i0 += CH) {
+          double2 y[CH][NJ][2];
 #pragma unroll
-          for (int j = 0; j < NJ; ++j)
+          for (int ii = 0; ii < CH; ++ii) {
+            const int m = S.m0 + wm * WTM + (i0 + ii) * 8 + (lane >> 2);
 #pragma unroll
-            for (int h = 0; h < 2; ++h) {
-              const int n = S.n0 + wn * WTN + j * 8 + (lane & 3) * 2 + h;
-              y[j][h] = (m < S.Mi && n < S.Ni) ? S.D[(long long)m * sDmi + (long long)n * sDni] : make_double2(0.0, 0.0);
-            }
+            for (int j = 0; j < NJ; ++j)
 #pragma unroll
-          for (int j = 0; j < NJ; ++j)
+              for (int h = 0; h < 2; ++h) {
+                const int n = S.n0 + wn * WTN + j * 8 + (lane & 3) * 2 + h;
+                y[ii][j][h] = (m < S.Mi && n < S.Ni) ? S.D[(long long)m * sDmi + (long long)n * sDni]
+                                                     : make_double2(0.0, 0.0);
+              }
+          }
 #pragma unroll
-            for (int h = 0; h < 2; ++h) {
-              double re, im;
-              cval(i, j, h, re, im);
-              pr += re * y[j][h].x - im * y[j][h].y;
-              pim += re * y[j][h].y + im * y[j][h].x;
-            }
+          for (int ii = 0; ii < CH; ++ii)
+#pragma unroll
+            for (int j = 0; j < NJ; ++j)
+#pragma unroll
+              for (int h = 0; h < 2; ++h) {
+                double re, im;
+                cval(i0 + ii, j, h, re, im);
+                pr += re * y[ii][j][h].x - im * y[ii][j][h].y;
+                pim += re * y[ii][j][h].y + im * y[ii][j][h].x;
+              }
         }
 #pragma unroll
         for (int off = 16; off > 0; off >>= 1) {
