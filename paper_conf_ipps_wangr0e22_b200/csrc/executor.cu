@@ -416,6 +416,8 @@ struct Executor::Impl {
       gemm_tile_shape(d.cls, &tbm, &tbn);
       d.tilesM = (L.Mi + tbm - 1) / tbm;
       d.tilesN = (L.Ni + tbn - 1) / tbn;
+      if ((long long)c.Lt * L.Mo * L.No * d.tilesM * d.tilesN >= (1LL << 32))
+        fail(MICCO_ERR_UNSUPPORTED, "executor: more than 2^32 tiles in one contraction");
       if (fd >= 0) {  // final dot in the epilogue: C is never materialised
         const TaskRec &dk = c.tasks[fd];
         const int32_t X = tk.out, Y = dk.a == X ? dk.b : dk.a;

@@ -226,8 +226,8 @@ __device__ __forceinline__ void decode_tile(const GemmDesc *__restrict__ descs, 
                                             long long tile, int tid, LoadCur<LPTA, LPTB> *L, StoreCur *S) {
   while (task + 1 < n_desc && descs[task + 1].tile_begin <= tile) ++task;
   const GemmDesc &d = descs[task];
-  long long lt = tile - d.tile_begin;
-  const int tilesN = d.tilesN, tilesM = d.tilesM, No = d.No, Mo = d.Mo;
+  unsigned lt = (unsigned)(tile - d.tile_begin);  // tiles of one task < 2^32: 32-bit div/mod
+  const unsigned tilesN = d.tilesN, tilesM = d.tilesM, No = d.No, Mo = d.Mo;
   const int tn = (int)(lt % tilesN); lt /= tilesN;
   const int tm = (int)(lt % tilesM); lt /= tilesM;
   const int no = (int)(lt % No); lt /= No;
