@@ -55,6 +55,8 @@ def parse():
     ap.add_argument("--dist", default="uniform", choices=["uniform", "gaussian"])
     ap.add_argument("--policy", default="micco")
     ap.add_argument("--window", type=int, default=0)
+    ap.add_argument("--reorder", action="store_true",
+                    help="reuse-aware reduction order (options.reorder, SURVEY.md §8(f) NEXT #3)")
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--cpu-sample", type=int, default=0, help="graphs in the oracle sample (0 = auto)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -198,7 +200,7 @@ def main():
     wl = c2_workload(args, world)
     t_setup = time.perf_counter()
     ctx = M.Context(keep_inputs_resident=True, policy=args.policy, window_graphs=args.window,
-                    dist_rank=rank if world > 1 else 0, dist_world=world if world > 1 else 0)
+                    reorder=args.reorder, dist_rank=rank if world > 1 else 0, dist_world=world if world > 1 else 0)
     if world > 1:
         obj = [M.micco_nccl_unique_id() if rank == 0 else None]
         dist.broadcast_object_list(obj, src=0)
@@ -300,6 +302,7 @@ def main():
                    "N": wl.meta.get("N", args.N), "Lt": wl.Lt,
                    "rate": args.rate if args.config == "c2" else None,
                    "dist": args.dist if args.config == "c2" else None, "policy": args.policy,
+                   "reduction_order": "reuse-aware (reorder)" if args.reorder else "as given",
                    "parallelism": f"task-parallel x{world} (MICCO scheduler)",
                    "l2": "inputs (node tensors) larger than L2; no flush",
                    "unique_gemms": s0["n_gemm"], "unique_dots": s0["n_dot"], "dedup_hits": s0["dedup_hits"],

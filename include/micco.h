@@ -94,6 +94,12 @@ typedef struct {
                                   released by micco_release_cache or destroy */
   int32_t dist_rank;           /* multi-process mode: this process's rank (one process per GPU); */
   int32_t dist_world;          /*   world size, 0 = single-process mode (default) */
+  int32_t reorder;             /* 1 = reuse-aware reduction order for every graph added from now on
+                                  (SURVEY.md §8(f) NEXT #3): the caller's order is ignored and each
+                                  step takes an already-interned contraction when one exists, else
+                                  the smallest result, fewest flops, fewest hadron nodes (so
+                                  node-pair products, the most shareable, come first), lowest
+                                  edge.  0 (default) = the caller's order, greedy when NULL */
 } micco_options;
 
 /* Fill *opt with the defaults (struct_size set). */

@@ -114,12 +114,18 @@ void build_graph(Context &ctx, int32_t n_inst, const int64_t *node_ids, int32_t 
     }
   }
 
-  // Two passes over the same decomposition: a dry run that validates ranks (so a failing
-  // graph leaves the DAG untouched), then the commit that interns tasks.
+  // Two passes over the same decomposition: a dry run that picks the steps and validates
+  // ranks and layouts (so a failing graph leaves the DAG untouched), then the commit that
+  // replays the dry run's steps and interns tasks.  The dry run predicts the ids the commit
+  // will give new tensors (they are appended in step order), so hash-consing keys — and the
+  // reuse-aware order, which looks them up — are identical in both passes.
+  const bool reorder = ctx.opt.reorder != 0;
+  std::vector<int32_t> chosen;  // edge picked at each step by the dry run
+  chosen.reserve(n_edges);
   for (int pass = 0; pass < 2; ++pass) {
     const bool commit = pass == 1;
     std::vector<Comp> comps(n_inst);
-    std::vector<int32_t> comp_of(n_inst);
+    std::vector<int32_t> comp_of(n_inst), n_members(n_inst, 1);
     for (int u = 0; u < n_inst; ++u) {
       Comp &c = comps[u];
       c.tensor = ctx.nodes[node_ids[u]].tensor;
@@ -132,6 +138,8 @@ void build_graph(Context &ctx, int32_t n_inst, const int64_t *node_ids, int32_t 
     std::vector<char> done(n_edges, 0);
     double flops_nd = 0;
     int steps_left = n_edges;
+    int32_t next_new = (int32_t)ctx.tensors.size();  // dry run: id the commit will assign
+    std::unordered_map<TaskKey, int32_t, TaskKeyHash> fresh;  // dry run: keys new in this graph
 
     auto plan_step = [&](int e, Step &st, int &res_rank, int64_t &res_size, int64_t &kdim) {
       const micco_edge &E = edges[e];
@@ -174,20 +182,53 @@ void build_graph(Context &ctx, int32_t n_inst, const int64_t *node_ids, int32_t 
       st.c = (int8_t)c;
       res_size = prod(comps[a].dim, comps[a].rank) * prod(comps[b].dim, comps[b].rank) / (kdim * kdim);
     };
+    // Canonical operand order for hash-consing: the lower tensor id is the left operand
+    // (a contraction and its mirror image are one task; the component keeps track of
+    // which legs the result carries, so the graph value is unchanged).
+    auto canonical = [&](Step &st) {
+      if (st.cb < 0 || comps[st.cb].tensor >= comps[st.ca].tensor) return;
+      std::swap(st.ca, st.cb);
+      int8_t pa2[kMaxRank], pb2[kMaxRank];
+      int idx[kMaxRank];
+      std::iota(idx, idx + st.c, 0);
+      std::sort(idx, idx + st.c, [&](int x, int y) { return st.pb[x] < st.pb[y]; });
+      for (int i = 0; i < st.c; ++i) { pa2[i] = st.pb[idx[i]]; pb2[i] = st.pa[idx[i]]; }
+      for (int i = 0; i < st.c; ++i) { st.pa[i] = pa2[i]; st.pb[i] = pb2[i]; }
+    };
+    auto make_key = [&](const Step &st) {
+      TaskKey key{};
+      key.a = comps[st.ca].tensor;
+      key.b = st.cb < 0 ? -1 : comps[st.cb].tensor;
+      key.c = st.c;
+      std::memcpy(key.pa, st.pa, kMaxRank);
+      std::memcpy(key.pb, st.pb, kMaxRank);
+      return key;
+    };
+    auto interned = [&](const TaskKey &key) {
+      return ctx.task_by_key.count(key) > 0 || (!commit && fresh.count(key) > 0);
+    };
 
     for (int step = 0; steps_left > 0; ++step) {
       int e = -1;
       Step st{};
       int rr = 0;
       int64_t rs = 0, kd = 0;
-      if (order) {
+      if (commit) {  // replay the dry run's choice
+        e = chosen[step];
+        plan_step(e, st, rr, rs, kd);
+      } else if (order && !reorder) {
         if (step >= n_edges) break;
         e = order[step];
         if (done[e]) continue;
         plan_step(e, st, rr, rs, kd);
-      } else {  // greedy: smallest result, then fewest flops, then lowest edge index
+      } else {
+        // greedy (order NULL): smallest result, then fewest flops, then lowest edge index.
+        // reuse-aware (options.reorder): an already-interned step first
+        // (free: dedup hit), then the same size/flops rule, then the fewest hadron nodes in
+        // the result — node-pair products are shared by the most graphs.
         int64_t best_s = 0;
         double best_f = 0;
+        int best_hit = 0, best_m = 0;
         for (int f = 0; f < n_edges; ++f) {
           if (done[f]) continue;
           Step s2{};
@@ -196,8 +237,17 @@ void build_graph(Context &ctx, int32_t n_inst, const int64_t *node_ids, int32_t 
           plan_step(f, s2, r2, sz, k2);
           if (r2 > kMaxRank) continue;
           double fl = (double)sz * (double)k2;
-          if (e < 0 || sz < best_s || (sz == best_s && fl < best_f)) {
-            e = f; st = s2; rr = r2; rs = sz; kd = k2; best_s = sz; best_f = fl;
+          int hit = 0, m = 0;
+          if (reorder) {
+            Step s3 = s2;
+            canonical(s3);
+            hit = interned(make_key(s3)) ? 0 : 1;
+            m = n_members[s2.ca] + (s2.cb >= 0 ? n_members[s2.cb] : 0);
+          }
+          bool better = e < 0 || hit < best_hit ||
+                        (hit == best_hit && (sz < best_s || (sz == best_s && (fl < best_f || (fl == best_f && m < best_m)))));
+          if (better) {
+            e = f; st = s2; rr = r2; rs = sz; kd = k2; best_s = sz; best_f = fl; best_hit = hit; best_m = m;
           }
         }
         if (e < 0) { plan_step(0, st, rr, rs, kd); rr = 99; }
@@ -216,6 +266,7 @@ void build_graph(Context &ctx, int32_t n_inst, const int64_t *node_ids, int32_t 
         }
         if (!ok) fail(MICCO_ERR_UNSUPPORTED, "add_graph: contraction layout not supported by the kernels");
       }
+      if (!commit) chosen.push_back(e);
       // mark contracted edges done
       {
         const micco_edge &E = edges[e];
@@ -228,18 +279,7 @@ void build_graph(Context &ctx, int32_t n_inst, const int64_t *node_ids, int32_t 
           if (hit) { done[f] = 1; --steps_left; }
         }
       }
-      // Canonical operand order for hash-consing: the lower tensor id is the left operand
-      // (a contraction and its mirror image are one task; the component keeps track of
-      // which legs the result carries, so the graph value is unchanged).
-      if (commit && st.cb >= 0 && comps[st.cb].tensor < comps[st.ca].tensor) {
-        std::swap(st.ca, st.cb);
-        int8_t pa2[kMaxRank], pb2[kMaxRank];
-        int idx[kMaxRank];
-        std::iota(idx, idx + st.c, 0);
-        std::sort(idx, idx + st.c, [&](int x, int y) { return st.pb[x] < st.pb[y]; });
-        for (int i = 0; i < st.c; ++i) { pa2[i] = st.pb[idx[i]]; pb2[i] = st.pa[idx[i]]; }
-        for (int i = 0; i < st.c; ++i) { st.pa[i] = pa2[i]; st.pb[i] = pb2[i]; }
-      }
+      canonical(st);
       Comp &A = comps[st.ca];
       Comp res{};
       res.alive = true;
@@ -267,13 +307,17 @@ void build_graph(Context &ctx, int32_t n_inst, const int64_t *node_ids, int32_t 
       }
       flops_nd += step_flops;
       res.tensor = -1;
-      if (commit) {
-        TaskKey key{};
-        key.a = A.tensor;
-        key.b = st.cb < 0 ? -1 : comps[st.cb].tensor;
-        key.c = st.c;
-        std::memcpy(key.pa, st.pa, kMaxRank);
-        std::memcpy(key.pb, st.pb, kMaxRank);
+      const TaskKey key = make_key(st);
+      if (!commit) {  // predict the id the commit gives this step's result
+        auto it = ctx.task_by_key.find(key);
+        if (it != ctx.task_by_key.end()) {
+          res.tensor = ctx.tasks[it->second].out;
+        } else {
+          auto jt = fresh.find(key);
+          if (jt != fresh.end()) res.tensor = jt->second;
+          else fresh.emplace(key, res.tensor = next_new++);
+        }
+      } else {
         auto it = ctx.task_by_key.find(key);
         if (it != ctx.task_by_key.end()) {
           res.tensor = ctx.tasks[it->second].out;
@@ -306,6 +350,7 @@ void build_graph(Context &ctx, int32_t n_inst, const int64_t *node_ids, int32_t 
       int ca = st.ca, cb = st.cb;
       comps[ca] = res;
       if (cb >= 0) {
+        n_members[ca] += n_members[cb];
         comps[cb].alive = false;
         for (int u = 0; u < n_inst; ++u)
           if (comp_of[u] == cb) comp_of[u] = ca;

@@ -201,9 +201,12 @@ Plan make_plan(const Context &ctx, const PlanInput &in) {
     }
   }
   // 1b. fuse a final dot into the GEMM that produces its operand when that product X is a
-  // matrix used by nothing else and the dot's other operand Y exists before the GEMM's
-  // stage: X is never written, Y is read in the GEMM epilogue (kernels.h GemmDesc::D).
-  // Decided from the DAG alone, so it is identical for every GPU count.
+  // matrix used by nothing else: X is never written, the dot's other operand Y is read in
+  // the GEMM epilogue (kernels.h GemmDesc::D), so the fused GEMM runs one stage after Y's
+  // producer at the earliest (plevel).  Decided from the DAG alone, so it is identical for
+  // every GPU count.
+  std::vector<int32_t> plevel(T);
+  for (int32_t t = 0; t < T; ++t) plevel[t] = ctx.tasks[t].level;
   plan.fused_dot.assign(T, -1);
   std::vector<char> skip(T, 0);
   std::vector<int32_t> extra(T, -1);  // fused GEMM task → Y
@@ -222,13 +225,14 @@ Plan make_plan(const Context &ctx, const PlanInput &in) {
         const int32_t pt = ctx.tensors[X].task;
         if (pt < 0 || consumers[X] != 1 || ctx.tensors[X].rank != 2) continue;
         const TaskRec &pk = ctx.tasks[pt];
-        if (pk.kind != TASK_GEMM || plan.fused_dot[pt] >= 0 || ctx.tensors[Y].level >= pk.level) continue;
+        if (pk.kind != TASK_GEMM || plan.fused_dot[pt] >= 0) continue;
         const TensorRec &A = ctx.tensors[pk.a], &B = ctx.tensors[pk.b];
         if (A.rank - pk.c != 1 || B.rank - pk.c != 1) continue;  // one M leg, one N leg
         GemmLayout L;
         if (!gemm_layout(A.rank, A.dim, B.rank, B.dim, pk.c, pk.pa, pk.pb, L) || gemm_class(L) == 4) continue;
         plan.fused_dot[pt] = d;
         extra[pt] = Y;
+        plevel[pt] = std::max(plevel[pt], ctx.tensors[Y].level + 1);
         skip[d] = 1;
         ++plan.n_fused;
         break;
@@ -251,13 +255,13 @@ Plan make_plan(const Context &ctx, const PlanInput &in) {
     if (task_window[t] >= 0 && !skip[t]) order.push_back(t);
   std::stable_sort(order.begin(), order.end(), [&](int32_t x, int32_t y) {
     if (task_window[x] != task_window[y]) return task_window[x] < task_window[y];
-    return ctx.tasks[x].level < ctx.tasks[y].level;
+    return plevel[x] < plevel[y];
   });
   std::vector<std::pair<int32_t, int32_t>> stages;  // [begin, end) in order
   for (size_t i = 0; i < order.size();) {
     size_t j = i;
     while (j < order.size() && task_window[order[j]] == task_window[order[i]] &&
-           ctx.tasks[order[j]].level == ctx.tasks[order[i]].level)
+           plevel[order[j]] == plevel[order[i]])
       ++j;
     stages.push_back({(int32_t)i, (int32_t)j});
     i = j;

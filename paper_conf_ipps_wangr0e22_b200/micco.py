@@ -35,7 +35,7 @@ class micco_options(ctypes.Structure):
     _fields_ = [("struct_size", ctypes.c_size_t), ("mem_budget_bytes", ctypes.c_int64),
                 ("policy", ctypes.c_int32), ("window_graphs", ctypes.c_int32), ("seed", ctypes.c_uint64),
                 ("deterministic", ctypes.c_int32), ("keep_inputs_resident", ctypes.c_int32),
-                ("dist_rank", ctypes.c_int32), ("dist_world", ctypes.c_int32)]
+                ("dist_rank", ctypes.c_int32), ("dist_world", ctypes.c_int32), ("reorder", ctypes.c_int32)]
 
 
 class micco_edge(ctypes.Structure):
@@ -136,7 +136,7 @@ def _check(ctx, st: int):
 
 def micco_create(mem_budget_bytes: int = 0, policy: str = "micco", window_graphs: int = 0,
                  keep_inputs_resident: bool = False, dist_rank: int = 0, dist_world: int = 0,
-                 deterministic: bool = True, seed: int = 0) -> ctypes.c_void_p:
+                 deterministic: bool = True, seed: int = 0, reorder: bool = False) -> ctypes.c_void_p:
     o = micco_options()
     lib().micco_options_default(ctypes.byref(o))
     o.mem_budget_bytes = int(mem_budget_bytes)
@@ -147,6 +147,7 @@ def micco_create(mem_budget_bytes: int = 0, policy: str = "micco", window_graphs
     o.dist_world = int(dist_world)
     o.deterministic = 1 if deterministic else 0
     o.seed = int(seed)
+    o.reorder = 1 if reorder else 0
     h = ctypes.c_void_p()
     _check(None, lib().micco_create(ctypes.byref(h), ctypes.byref(o)))
     return h

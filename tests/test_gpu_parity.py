@@ -189,3 +189,23 @@ def test_c5_mixed_oversubscribed():
     assert st["evictions"] > 0 and st["bytes_d2h"] > 0 and st["bytes_p2p"] > 0, st
     ref, _, _ = run_gpu(wl, 1)
     assert np.array_equal(C, ref)
+
+
+def test_reorder_parity():
+    """Reuse-aware reduction order (options.reorder): the caller's
+    order is replaced, the values are not — against the oracle (which contracts in the
+    caller's order) on C3 wirings, random meson/baryon graphs and C4 chain graphs, bit-exact
+    on integer inputs, and bitwise identical across GPU counts."""
+    check(workloads.c3_multi_meson(n_graphs=60, N=40, Lt=3, pool=4), reorder=True)
+    check(workloads.tiny_random(seed=7, n_graphs=40, N=3, Lt=2), reorder=True)
+    check(workloads.c4_two_baryon(n_combos=1, N=9, Lt=2, pool=2, order="chain"), reorder=True)
+    wli = workloads.c3_multi_meson(n_graphs=60, N=40, Lt=2, pool=4, mode=MODE_INT3)
+    _, vals, _ = run_gpu(wli, reorder=True)
+    _, valso = oracle.correlator(wli, return_values=True)
+    assert np.array_equal(vals, valso)
+    wl = workloads.c2_meson_set(n_graphs=120, N=24, Lt=4, rate=0.6, dist="gaussian", flips=True)
+    ref, _, _ = run_gpu(wl, 1, reorder=True)
+    assert rel_err(ref, oracle.correlator(wl)) <= TOL
+    for n in (2, 4):
+        C, _, _ = run_gpu(wl, n, [1, 2, 0], reorder=True, window_graphs=16)
+        assert np.array_equal(C, ref), n

@@ -203,3 +203,45 @@ def test_native_scheduler_matches_oracle(seed):
     got_o = O.run([[Pair(*p) for p in v] for v in vecs])
     got_n = M.micco_debug_schedule(n, bd, budget, vecs, resident=res)
     assert got_n == got_o
+
+
+def test_reorder_reuse_aware_dedup():
+    """options.reorder: on the C3 wiring the node-pair products
+    S·R come first and are shared by many graphs, so the unique GEMMs drop > 2x (3.5x at 10k graphs) against
+    the chain order; on C4 the chain order collapses to the greedy (c = 2 first) DAG; the
+    graph count and the flops of the as-given DAG are unchanged by construction."""
+    wl = workloads.c3_multi_meson(n_graphs=2000, N=4, Lt=1)
+    counts = {}
+    for reorder in (False, True):
+        ctx = _ctx(reorder=reorder)
+        M.load_workload(ctx, wl)
+        st, _ = ctx.plan(1, [0, 0, 0])
+        counts[reorder] = st
+        ctx.close()
+    assert counts[True]["n_gemm"] * 2 < counts[False]["n_gemm"], (counts[True]["n_gemm"], counts[False]["n_gemm"])
+    assert counts[True]["flops"] < counts[False]["flops"]
+    assert counts[True]["flops_no_dedup"] > 0
+    c4 = {}
+    for order, reorder in (("greedy", False), ("chain", False), ("chain", True)):
+        ctx = _ctx(reorder=reorder)
+        M.load_workload(ctx, workloads.c4_two_baryon(n_combos=4, N=3, Lt=1, order=order))
+        c4[(order, reorder)] = ctx.plan(1, [0, 0, 0])[0]
+        ctx.close()
+    assert c4[("chain", True)]["n_gemm"] == c4[("greedy", False)]["n_gemm"] < c4[("chain", False)]["n_gemm"]
+
+
+def test_reorder_dry_run_leaves_dag_untouched_on_failure():
+    """The dry pass predicts tensor ids exactly; a graph that fails validation under
+    reorder leaves no task behind."""
+    ctx = _ctx(reorder=True)
+    rng = np.random.default_rng(3)
+    ids = [ctx.add_node(rng.standard_normal((1, 4, 4)) + 0j) for _ in range(3)]
+    ctx.add_graph(ids, workloads.meson_cycle_edges(3), None)
+    st0, _ = ctx.plan(1, [0, 0, 0])
+    with pytest.raises(M.MiccoError):
+        ctx.add_graph(ids, [(0, 1, 1, 0), (1, 1, 2, 0), (2, 1, 2, 0)], None)  # leg (2, 0) twice
+    st1, _ = ctx.plan(1, [0, 0, 0])
+    assert st1["unique_tasks"] == st0["unique_tasks"]
+    ctx.add_graph([ids[1], ids[2], ids[0]], workloads.meson_cycle_edges(3), None)  # rotation: all hits
+    st2, _ = ctx.plan(1, [0, 0, 0])
+    assert st2["unique_tasks"] == st0["unique_tasks"] and st2["dedup_hits"] == st0["dedup_hits"] + 2

@@ -97,3 +97,15 @@ def test_replay_keep_inputs_and_fusion():
     ops, fused = M.micco_plan_ops(ctx.h, 1, [0, 0, 0])
     assert (fused >= 0).sum() > 0  # most cycles end in a fused GEMM → dot
     replay(ctx, 1, [0, 0, 0], 1 << 30)
+
+
+@pytest.mark.parametrize("n_gpus", [1, 3])
+def test_replay_reorder_c3(n_gpus):
+    """Reuse-aware order: final dots of two level-1 products are fused into the later GEMM
+    (its stage moves after the partner's producer); replay checks the partner is resident."""
+    wl = workloads.c3_multi_meson(n_graphs=400, N=4, Lt=1, pool=6)
+    ctx = M.Context(mem_budget_bytes=1 << 30, reorder=True, window_graphs=64)
+    M.load_workload(ctx, wl)
+    ops, fused = M.micco_plan_ops(ctx.h, n_gpus, [1, 1, 0])
+    assert (fused >= 0).sum() > 0
+    replay(ctx, n_gpus, [1, 1, 0], 1 << 30)
