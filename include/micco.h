@@ -100,6 +100,13 @@ typedef struct {
                                   the smallest result, fewest flops, fewest hadron nodes (so
                                   node-pair products, the most shareable, come first), lowest
                                   edge.  0 (default) = the caller's order, greedy when NULL */
+  int32_t bound_model;         /* how execute(reuse_bound = NULL) picks the reuse bounds on more than
+                                  one GPU: 0 (default) one set for the whole plan, the cheapest of
+                                  {0,1,2}^3 under the planner's cost model; 1 a set per vector
+                                  (stage), the cheapest for that vector; 2 a set per vector from the
+                                  fitted regression (a random forest over vector
+                                  features, trained offline on mode-1 choices by
+                                  tools/train_bounds.py) */
 } micco_options;
 
 /* Fill *opt with the defaults (struct_size set). */
@@ -227,6 +234,23 @@ MICCO_API micco_status micco_plan(micco_ctx *ctx, int32_t n_gpus, const int32_t 
  * receives, per task, the dot task fused into its epilogue or −1. */
 MICCO_API micco_status micco_plan_ops(micco_ctx *ctx, int32_t n_gpus, const int32_t *reuse_bound,
                                       int64_t max_ops, int32_t *ops, int64_t *n_ops, int32_t *fused);
+
+/* Per-vector reuse bounds.  Plans like micco_plan with bound_mode 0
+ * (reuse_bound, or the whole-plan sweep when NULL), 1 (per-vector sweep) or 2 (per-vector
+ * regression); copies, for up to max_stages stages in order, the 6 vector features (balanceNum =
+ * ceil(pairs/n_gpus), log2 mean operand bytes, repeated rate, resident rate, n_gpus, memory
+ * pressure = max resident/budget; taken before the vector is scheduled) into features[6*s..]
+ * and the bounds used into bounds[3*s..].  *n_stages receives the stage count, *predicted_s
+ * the plan's modelled time (max over GPUs per stage of flops/30 TF/s + host bytes/55 GB/s +
+ * peer bytes/700 GB/s, summed over stages).  Needs options.mem_budget_bytes; no GPU. */
+MICCO_API micco_status micco_plan_stages(micco_ctx *ctx, int32_t n_gpus, int32_t bound_mode,
+                                         const int32_t *reuse_bound, int64_t max_stages,
+                                         double *features, int32_t *bounds, int64_t *n_stages,
+                                         double *predicted_s);
+
+/* The fitted reuse-bound regression on one 6-feature vector (layout as micco_plan_stages):
+ * raw[3] receives the forest's mean output, bounds[3] the rounded values clamped to [0, 2]. */
+MICCO_API void micco_predict_bounds(const double *features, double *raw, int32_t *bounds);
 
 /* The task DAG: per tensor its size in bytes (all Lt slices; 0 for per-slice scalars) and its
  * producing task (−1 for hadron nodes); per task (kind 0 GEMM / 1 dot / 2 trace, operand a,

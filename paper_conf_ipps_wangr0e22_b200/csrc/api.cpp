@@ -161,7 +161,7 @@ MICCO_API micco_status micco_create(micco_ctx **out, const micco_options *opt) {
     o.struct_size = sizeof(o);
   }
   if (o.policy < 0 || o.policy > 3 || o.window_graphs < 0 || o.mem_budget_bytes < 0 || o.dist_world < 0 ||
-      o.reorder < 0 || o.reorder > 1 ||
+      o.reorder < 0 || o.reorder > 1 || o.bound_model < 0 || o.bound_model > 2 ||
       (o.dist_world > 0 && (o.dist_rank < 0 || o.dist_rank >= o.dist_world)))
     return MICCO_ERR_ARG;
   micco_ctx *c = new (std::nothrow) micco_ctx;
@@ -302,7 +302,7 @@ MICCO_API micco_status micco_execute(micco_ctx *ctx, int32_t n_gpus, const int32
 }
 
 namespace {
-Plan host_plan(Context &c, int32_t n_gpus, const int32_t *reuse_bound) {
+Plan host_plan(Context &c, int32_t n_gpus, const int32_t *reuse_bound, int32_t bound_mode = -1) {
   if (n_gpus < 1 || n_gpus > 64) fail(MICCO_ERR_ARG, "n_gpus must be in [1, 64]");
   if (c.opt.mem_budget_bytes <= 0) fail(MICCO_ERR_ARG, "micco_plan needs options.mem_budget_bytes");
   PlanInput in;
@@ -315,9 +315,41 @@ Plan host_plan(Context &c, int32_t n_gpus, const int32_t *reuse_bound) {
   in.peer_gbs = 700;
   in.host_gbs = 55;
   in.flops_per_s = 30e12;
+  if (bound_mode < 0) bound_mode = reuse_bound ? BOUNDS_FIXED : c.opt.bound_model;
+  if (bound_mode != BOUNDS_FIXED) {
+    in.bound_mode = bound_mode;
+    return make_plan(c, in);
+  }
   return reuse_bound ? make_plan(c, in) : make_plan_auto(c, in);
 }
 }  // namespace
+
+MICCO_API micco_status micco_plan_stages(micco_ctx *ctx, int32_t n_gpus, int32_t bound_mode,
+                                         const int32_t *reuse_bound, int64_t max_stages, double *features,
+                                         int32_t *bounds, int64_t *n_stages, double *predicted_s) {
+  return guard(ctx, [&] {
+    if (bound_mode < 0 || bound_mode > 2) fail(MICCO_ERR_ARG, "bound_mode must be 0, 1 or 2");
+    Plan p = host_plan(ctx->c, n_gpus, reuse_bound, bound_mode);
+    const int64_t ns = (int64_t)p.stage_bounds.size() / 3;
+    if (n_stages) *n_stages = ns;
+    if (predicted_s) *predicted_s = p.predicted_s;
+    const int64_t k = std::min(max_stages, ns);
+    if (features) std::copy(p.stage_features.begin(), p.stage_features.begin() + k * kBoundFeatures, features);
+    if (bounds) std::copy(p.stage_bounds.begin(), p.stage_bounds.begin() + k * 3, bounds);
+  });
+}
+
+MICCO_API void micco_predict_bounds(const double *features, double *raw, int32_t *bounds) {
+  if (!features) return;
+  int32_t b[3];
+  double r[3];
+  predict_bounds_raw(features, r);
+  predict_bounds(features, b);
+  for (int i = 0; i < 3; ++i) {
+    if (raw) raw[i] = r[i];
+    if (bounds) bounds[i] = b[i];
+  }
+}
 
 MICCO_API micco_status micco_plan_ops(micco_ctx *ctx, int32_t n_gpus, const int32_t *reuse_bound, int64_t max_ops,
                                       int32_t *ops, int64_t *n_ops, int32_t *fused) {

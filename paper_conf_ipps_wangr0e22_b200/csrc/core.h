@@ -193,7 +193,22 @@ struct Plan {
   std::vector<std::pair<int32_t, uint64_t>> final_nodes;  // (node tensor, GPU mask) left cached
   std::vector<int32_t> fused_dot;  // GEMM task → DOT task fused into its epilogue, or -1
   int64_t n_fused = 0;
+  std::vector<double> stage_features;  // kBoundFeatures per stage (planner.cpp stage_features)
+  std::vector<int32_t> stage_bounds;   // reuse bounds used per stage (3 each)
 };
+
+// Per-vector features of the reuse-bound model (vector size, tensor size,
+// distribution, repeated rate), computed at the start of each stage:
+//   0 balanceNum = ceil(pairs / n_gpus)      1 log2(mean operand bytes)
+//   2 repeated rate (operand slots whose tensor occurs twice or more in the vector)
+//   3 resident rate (operand slots already resident on some GPU: the locality a Gaussian
+//     selection gives, L314)                  4 n_gpus
+//   5 memory pressure max_g resident / budget
+constexpr int kBoundFeatures = 6;
+// bound_mode: how each stage's reuse bounds are chosen
+enum { BOUNDS_FIXED = 0, BOUNDS_STAGE_SWEEP = 1, BOUNDS_REGRESSION = 2 };
+void predict_bounds(const double *features, int32_t out[3]);  // bounds_model.cpp
+void predict_bounds_raw(const double *features, double out[3]);
 
 struct PlanInput {
   int32_t n_gpus;
@@ -205,6 +220,7 @@ struct PlanInput {
   bool fuse = true;                                 // fuse GEMM → final dot when legal
   std::vector<std::vector<int32_t>> initial_nodes;  // per GPU: node tensors already resident
   double peer_gbs, host_gbs, flops_per_s;           // cost model of the bound sweep
+  int32_t bound_mode = BOUNDS_FIXED;                // per-stage bounds (BOUNDS_*)
 };
 
 Plan make_plan(const Context &ctx, const PlanInput &in);

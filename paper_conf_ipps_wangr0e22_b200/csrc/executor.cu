@@ -635,7 +635,11 @@ struct Executor::Impl {
             in.initial_nodes[i].push_back(fn.first);
           }
     Plan plan;
-    if (bd) {
+    if (!bd && c.opt.bound_model != BOUNDS_FIXED) {  // per-vector bounds (sweep or regression)
+      in.bound_mode = c.opt.bound_model;
+      for (int i = 0; i < 3; ++i) in.reuse_bound[i] = 0;
+      plan = make_plan(c, in);
+    } else if (bd) {
       for (int i = 0; i < 3; ++i) in.reuse_bound[i] = bd[i];
       plan = make_plan(c, in);
     } else if (chosen_bd_n == n) {  // bounds chosen by an earlier sweep for this GPU count

@@ -304,8 +304,9 @@ Plan make_plan(const Context &ctx, const PlanInput &in) {
     ++S.epoch[g];
   };
 
-  double predicted = 0;
-  for (int32_t s = 0; s < (int32_t)stages.size(); ++s) {
+  // One stage (a vector of independent pairs): schedule, simulate the cache, emit the ops,
+  // release dead operands.  Returns the stage's modelled time (max over GPUs).
+  auto run_stage = [&](int32_t s) -> double {
     S.stage = s;
     sched.begin_vector(stages[s].second - stages[s].first);
     std::fill(S.st_flops.begin(), S.st_flops.end(), 0.0);
@@ -382,7 +383,93 @@ Plan make_plan(const Context &ctx, const PlanInput &in) {
                   S.st_p2p[g] / (in.peer_gbs * 1e9);
       worst = std::max(worst, tg);
     }
-    predicted += worst;
+    return worst;
+  };
+
+  // Per-vector features (core.h kBoundFeatures), from the state before the stage runs.
+  auto stage_features = [&](int32_t s, double *f) {
+    int64_t slots = 0, repeated = 0, resident = 0;
+    double bytes = 0;
+    std::vector<int32_t> seen;
+    for (int32_t i = stages[s].first; i < stages[s].second; ++i) {
+      int32_t ops[3];
+      const int k = operands(order[i], ops);
+      for (int j = 0; j < k; ++j) seen.push_back(ops[j]);
+    }
+    std::vector<int32_t> sorted = seen;
+    std::sort(sorted.begin(), sorted.end());
+    for (int32_t x : seen) {
+      ++slots;
+      bytes += (double)S.bytes(x);
+      auto r = std::equal_range(sorted.begin(), sorted.end(), x);
+      if (r.second - r.first >= 2) ++repeated;
+      if (S.mask[x]) ++resident;
+    }
+    const int64_t pairs = stages[s].second - stages[s].first;
+    double pressure = 0;
+    for (int g = 0; g < n; ++g) pressure = std::max(pressure, (double)S.mem[g] / (double)in.budget[g]);
+    f[0] = (double)((pairs + n - 1) / n);
+    f[1] = std::log2(std::max(1.0, bytes / std::max<int64_t>(1, slots)));
+    f[2] = slots ? (double)repeated / (double)slots : 0.0;
+    f[3] = slots ? (double)resident / (double)slots : 0.0;
+    f[4] = (double)n;
+    f[5] = pressure;
+  };
+
+  // Snapshot of everything a stage mutates, for the per-stage bound sweep.
+  struct Snap {
+    std::vector<uint64_t> mask;
+    std::vector<char> on_host;
+    std::vector<int32_t> uses_left, epoch;
+    std::vector<std::vector<int32_t>> res, res_pos, pin;
+    std::vector<int64_t> mem, peak;
+    std::vector<double> gpu_flops;
+    size_t n_ops;
+    int64_t h2d, p2p, d2h, ev, hits;
+    double flops;
+  };
+  auto save = [&](Snap &z) {
+    z.mask = S.mask; z.on_host = S.on_host; z.uses_left = S.uses_left; z.epoch = S.epoch;
+    z.res = S.res; z.res_pos = S.res_pos; z.pin = S.pin; z.mem = S.mem; z.peak = plan.gpu_peak_bytes;
+    z.gpu_flops = plan.gpu_flops; z.n_ops = plan.ops.size();
+    z.h2d = plan.bytes_h2d; z.p2p = plan.bytes_p2p; z.d2h = plan.bytes_d2h; z.ev = plan.evictions;
+    z.hits = plan.cache_hits; z.flops = plan.flops;
+  };
+  auto restore = [&](const Snap &z) {
+    S.mask = z.mask; S.on_host = z.on_host; S.uses_left = z.uses_left; S.epoch = z.epoch;
+    S.res = z.res; S.res_pos = z.res_pos; S.pin = z.pin; S.mem = z.mem; plan.gpu_peak_bytes = z.peak;
+    plan.gpu_flops = z.gpu_flops; plan.ops.resize(z.n_ops);
+    plan.bytes_h2d = z.h2d; plan.bytes_p2p = z.p2p; plan.bytes_d2h = z.d2h; plan.evictions = z.ev;
+    plan.cache_hits = z.hits; plan.flops = z.flops;
+  };
+
+  const bool per_stage = in.bound_mode != BOUNDS_FIXED && n > 1 && in.policy == MICCO_POLICY_MICCO;
+  double predicted = 0;
+  for (int32_t s = 0; s < (int32_t)stages.size(); ++s) {
+    double f[kBoundFeatures];
+    stage_features(s, f);
+    plan.stage_features.insert(plan.stage_features.end(), f, f + kBoundFeatures);
+    int32_t bd[3] = {in.reuse_bound[0], in.reuse_bound[1], in.reuse_bound[2]};
+    if (per_stage && in.bound_mode == BOUNDS_REGRESSION) {
+      predict_bounds(f, bd);
+    } else if (per_stage) {  // BOUNDS_STAGE_SWEEP: try {0,1,2}^3 on this stage, keep the cheapest
+      Snap z;
+      save(z);
+      const Scheduler sched0 = sched;
+      double best = 0;
+      bool have = false;
+      for (int c = 0; c < 27; ++c) {
+        const int32_t cand[3] = {c / 9, (c / 3) % 3, c % 3};
+        sched.set_bounds(cand);
+        const double cost = run_stage(s);
+        if (!have || cost < best * (1 - 1e-12)) { best = cost; have = true; for (int i = 0; i < 3; ++i) bd[i] = cand[i]; }
+        restore(z);
+        sched = sched0;
+      }
+    }
+    sched.set_bounds(bd);
+    plan.stage_bounds.insert(plan.stage_bounds.end(), bd, bd + 3);
+    predicted += run_stage(s);
   }
   if (in.keep_inputs)
     for (int32_t x = 0; x < NT; ++x)

@@ -11,6 +11,10 @@ Scheduler::Scheduler(int n_gpus, int policy, const int32_t bd[3], std::vector<in
   for (int i = 0; i < 3; ++i) bd_[i] = (policy == MICCO_POLICY_MICCO_NAIVE) ? 0 : bd[i];
 }
 
+void Scheduler::set_bounds(const int32_t bd[3]) {
+  for (int i = 0; i < 3; ++i) bd_[i] = (policy_ == MICCO_POLICY_MICCO_NAIVE) ? 0 : bd[i];
+}
+
 void Scheduler::begin_vector(int64_t num_pairs) {
   balance_ = (num_pairs + n - 1) / n;  // balanceNum, reading #14
   std::fill(count_.begin(), count_.end(), 0);

@@ -36,6 +36,8 @@ class Scheduler {
   int decide(const SchedPair &p);
   // line 20 bookkeeping that is not residency: count, com (and cumulative load)
   void account(int g, const SchedPair &p);
+  // reuseBd for the next vectors (per-vector bounds)
+  void set_bounds(const int32_t bd[3]);
   std::vector<int64_t> mem;   // mapGPUMem, maintained by the caller
   int n;
  private:

@@ -35,7 +35,8 @@ class micco_options(ctypes.Structure):
     _fields_ = [("struct_size", ctypes.c_size_t), ("mem_budget_bytes", ctypes.c_int64),
                 ("policy", ctypes.c_int32), ("window_graphs", ctypes.c_int32), ("seed", ctypes.c_uint64),
                 ("deterministic", ctypes.c_int32), ("keep_inputs_resident", ctypes.c_int32),
-                ("dist_rank", ctypes.c_int32), ("dist_world", ctypes.c_int32), ("reorder", ctypes.c_int32)]
+                ("dist_rank", ctypes.c_int32), ("dist_world", ctypes.c_int32), ("reorder", ctypes.c_int32),
+                ("bound_model", ctypes.c_int32)]
 
 
 class micco_edge(ctypes.Structure):
@@ -69,7 +70,7 @@ EXPORTS = ["micco_options_default", "micco_create", "micco_destroy", "micco_add_
            "micco_add_hadron_nodes_synth", "micco_add_graph", "micco_execute", "micco_get_correlator",
            "micco_get_graph_value", "micco_last_error", "micco_get_stats", "micco_release_cache",
            "micco_nccl_unique_id", "micco_set_nccl_id", "micco_plan", "micco_plan_ops", "micco_dag",
-           "micco_debug_schedule"]
+           "micco_debug_schedule", "micco_plan_stages", "micco_predict_bounds"]
 
 _lib = None
 
@@ -112,7 +113,11 @@ def lib() -> ctypes.CDLL:
         L.micco_debug_schedule.argtypes = [ctypes.c_int32, P(ctypes.c_int32), ctypes.c_double, ctypes.c_int32,
                                            P(ctypes.c_int64), P(ctypes.c_double), ctypes.c_int32,
                                            P(ctypes.c_int64), P(ctypes.c_int32)]
-        for f in ("micco_create", "micco_add_hadron_node", "micco_add_hadron_nodes_synth", "micco_add_graph",
+        L.micco_plan_stages.argtypes = [vp, ctypes.c_int32, ctypes.c_int32, P(ctypes.c_int32), ctypes.c_int64,
+                                        P(ctypes.c_double), P(ctypes.c_int32), P(ctypes.c_int64), P(ctypes.c_double)]
+        L.micco_predict_bounds.argtypes = [P(ctypes.c_double), P(ctypes.c_double), P(ctypes.c_int32)]
+        L.micco_predict_bounds.restype = None
+        for f in ("micco_plan_stages", "micco_create", "micco_add_hadron_node", "micco_add_hadron_nodes_synth", "micco_add_graph",
                   "micco_execute", "micco_get_correlator", "micco_get_graph_value", "micco_get_stats",
                   "micco_release_cache", "micco_nccl_unique_id", "micco_set_nccl_id", "micco_plan",
                   "micco_plan_ops", "micco_dag", "micco_debug_schedule"):
@@ -136,7 +141,8 @@ def _check(ctx, st: int):
 
 def micco_create(mem_budget_bytes: int = 0, policy: str = "micco", window_graphs: int = 0,
                  keep_inputs_resident: bool = False, dist_rank: int = 0, dist_world: int = 0,
-                 deterministic: bool = True, seed: int = 0, reorder: bool = False) -> ctypes.c_void_p:
+                 deterministic: bool = True, seed: int = 0, reorder: bool = False,
+                 bound_model: int = 0) -> ctypes.c_void_p:
     o = micco_options()
     lib().micco_options_default(ctypes.byref(o))
     o.mem_budget_bytes = int(mem_budget_bytes)
@@ -148,6 +154,7 @@ def micco_create(mem_budget_bytes: int = 0, policy: str = "micco", window_graphs
     o.deterministic = 1 if deterministic else 0
     o.seed = int(seed)
     o.reorder = 1 if reorder else 0
+    o.bound_model = int(bound_model)
     h = ctypes.c_void_p()
     _check(None, lib().micco_create(ctypes.byref(h), ctypes.byref(o)))
     return h
@@ -249,6 +256,33 @@ def micco_plan_ops(ctx, n_gpus: int, reuse_bound: Optional[Sequence[int]] = None
     _check(ctx, lib().micco_plan_ops(ctx, int(n_gpus), bd, n.value, _ptr(ops, ctypes.c_int32), ctypes.byref(n),
                                      _ptr(fused, ctypes.c_int32)))
     return ops[:n.value], fused[:nt.value]
+
+
+BOUND_MODES = {"fixed": 0, "stage_sweep": 1, "regression": 2}
+
+
+def micco_plan_stages(ctx, n_gpus: int, bound_mode, reuse_bound: Optional[Sequence[int]] = None):
+    """(features[n_stages, 6], bounds[n_stages, 3], predicted_s) of the plan under bound_mode
+    ('fixed' | 'stage_sweep' | 'regression' or 0/1/2)."""
+    mode = BOUND_MODES[bound_mode] if isinstance(bound_mode, str) else int(bound_mode)
+    bd = None if reuse_bound is None else (ctypes.c_int32 * 3)(*[int(x) for x in reuse_bound])
+    ns, pred = ctypes.c_int64(), ctypes.c_double()
+    _check(ctx, lib().micco_plan_stages(ctx, int(n_gpus), mode, bd, 0, None, None, ctypes.byref(ns),
+                                        ctypes.byref(pred)))
+    f = np.zeros((max(1, ns.value), 6))
+    b = np.zeros((max(1, ns.value), 3), dtype=np.int32)
+    _check(ctx, lib().micco_plan_stages(ctx, int(n_gpus), mode, bd, ns.value, _ptr(f, ctypes.c_double),
+                                        _ptr(b, ctypes.c_int32), ctypes.byref(ns), ctypes.byref(pred)))
+    return f[:ns.value], b[:ns.value], pred.value
+
+
+def micco_predict_bounds(features: Sequence[float]):
+    """(raw[3], bounds[3]) of the fitted reuse-bound regression on one feature vector."""
+    f = np.ascontiguousarray(np.asarray(features, dtype=np.float64).reshape(6))
+    raw = np.zeros(3)
+    b = np.zeros(3, dtype=np.int32)
+    lib().micco_predict_bounds(_ptr(f, ctypes.c_double), _ptr(raw, ctypes.c_double), _ptr(b, ctypes.c_int32))
+    return raw, b
 
 
 def micco_dag(ctx):

@@ -115,6 +115,9 @@ def test_cross_run_invariance_bitwise():
     for bd in ([0, 0, 0], [2, 2, 2], None):
         C, _, _ = run_gpu(wl, 4, bd)
         assert np.array_equal(C, ref)
+    for bm in (1, 2):  # per-vector bounds: sweep, regression
+        C, _, _ = run_gpu(wl, 4, None, bound_model=bm, window_graphs=16)
+        assert np.array_equal(C, ref), bm
     # memory pressure: evictions and host spills
     C, _, st = run_gpu(wl, 2, [1, 1, 1], mem_budget_bytes=10 * node_bytes, window_graphs=40)
     assert st["evictions"] > 0
