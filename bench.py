@@ -46,7 +46,7 @@ def parse():
     ap.add_argument("--steps", type=int, default=5)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="micco", choices=["micco", "reference"])
-    ap.add_argument("--config", default="c2", choices=["c2", "c3", "c4"],
+    ap.add_argument("--config", default="c2", choices=["c2", "c3", "c4", "c5"],
                     help="c2 = BASELINE configs[1] (the headline); c3 / c4 = configs[2] / [3] shapes")
     ap.add_argument("--graphs", type=int, default=10000, help="graphs per GPU (weak scaling)")
     ap.add_argument("--N", type=int, default=128)
@@ -55,6 +55,9 @@ def parse():
     ap.add_argument("--dist", default="uniform", choices=["uniform", "gaussian"])
     ap.add_argument("--policy", default="micco")
     ap.add_argument("--window", type=int, default=0)
+    ap.add_argument("--budget-gb", type=float, default=0.0,
+                    help="per-GPU memory budget (0 = device free memory; c5 defaults to 25 GB: its "
+                         "unconstrained plan peaks at 37.6 GB, so demand/budget = 150%%, PAPER.md L376)")
     ap.add_argument("--reorder", action="store_true",
                     help="reuse-aware reduction order (options.reorder, SURVEY.md §8(f) NEXT #3)")
     ap.add_argument("--e2e-steps", type=int, default=2)
@@ -114,6 +117,10 @@ def c2_workload(args, world):
     from micco_inputs import workloads
     if args.config == "c3":  # multi-meson: N = 256, Lt = 128 (BASELINE configs[2])
         return workloads.c3_multi_meson(n_graphs=args.graphs * world, N=256, Lt=128)
+    if args.config == "c5":  # oversubscribed mixed set (configs[4]), scaled to the host's RAM:
+        # rank-4 N = 64 intermediates of 4.3 GB (Lt = 16) shared across the stream, plus C3-style
+        # N = 256 meson graphs; unconstrained peak 37.6 GB, run against a 25 GB budget
+        return workloads.c5_mixed(n_combos=1, Nb=64, Nm=256, Lt=16, pool=2, meson_graphs=64)
     if args.config == "c4":  # two-baryon: rank-3 N = 64, Lt = 64 (configs[3]); graphs = combos × 720
         return workloads.c4_two_baryon(n_combos=max(1, args.graphs * world // 720), N=64, Lt=64, order="greedy")
     return workloads.c2_meson_set(n_graphs=args.graphs * world, N=args.N, Lt=args.Lt, rate=args.rate,
@@ -199,7 +206,9 @@ def main():
 
     wl = c2_workload(args, world)
     t_setup = time.perf_counter()
+    budget_gb = args.budget_gb or (25.0 if args.config == "c5" else 0.0)
     ctx = M.Context(keep_inputs_resident=True, policy=args.policy, window_graphs=args.window,
+                    mem_budget_bytes=int(budget_gb * 1e9),
                     reorder=args.reorder, dist_rank=rank if world > 1 else 0, dist_world=world if world > 1 else 0)
     if world > 1:
         obj = [M.micco_nccl_unique_id() if rank == 0 else None]
@@ -303,11 +312,13 @@ def main():
                    "rate": args.rate if args.config == "c2" else None,
                    "dist": args.dist if args.config == "c2" else None, "policy": args.policy,
                    "reduction_order": "reuse-aware (reorder)" if args.reorder else "as given",
+                   "budget_gb": budget_gb or None,
                    "parallelism": f"task-parallel x{world} (MICCO scheduler)",
                    "l2": "inputs (node tensors) larger than L2; no flush",
                    "unique_gemms": s0["n_gemm"], "unique_dots": s0["n_dot"], "dedup_hits": s0["dedup_hits"],
                    "setup_s": round(t_setup, 1)},
         "tflops": flops_step / (ms_per_step / 1e3) / 1e12,
+        "cache_per_step": {k: s0[k] for k in ("evictions", "cache_hits", "bytes_h2d", "bytes_d2h", "bytes_p2p")},
         "roofline": {"bound": "tensor", "kernel": "zgemm_dmma_kernel (grouped)", "achieved": achieved,
                      "peak": FP64_DMMA_PEAK_TFLOPS, "unit": "TFLOP/s", "frac": achieved / FP64_DMMA_PEAK_TFLOPS,
                      "peak_source": "measured FP64 DMMA microbenchmark (profiles/fp64_peak_r01.txt); "

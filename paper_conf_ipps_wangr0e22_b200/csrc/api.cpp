@@ -30,18 +30,19 @@ void HostArena::release_all() {
   }
   chunks_.clear();
   cur_ = 0;
-  for (auto &b : big_) {
-    if (b.second) cudaFreeHost(b.first); else std::free(b.first);
+  rewind();
+  for (auto &kv : big_free_) {
+    if (kv.second.pinned) cudaFreeHost(kv.second.base); else std::free(kv.second.base);
   }
-  big_.clear();
+  big_free_.clear();
 }
 
 void HostArena::rewind() {
   for (auto &c : chunks_) c.used = 0;
   cur_ = 0;
-  for (auto &b : big_) {
-    if (b.second) cudaFreeHost(b.first); else std::free(b.first);
-  }
+  // large blocks go back to a free list: pinning gigabytes costs ~0.5 s/GB, so an execute that
+  // spills rank-4 intermediates would otherwise re-pin them every time
+  for (auto &b : big_) big_free_.emplace(b.size, b);
   big_.clear();
 }
 
@@ -61,10 +62,17 @@ double *HostArena::alloc(int64_t bytes) {
     return (char *)p;
   };
   if (bytes > kChunk / 4) {
+    auto it = big_free_.lower_bound(bytes);  // smallest kept block that fits, if not wasteful
+    if (it != big_free_.end() && it->first <= bytes + bytes / 4) {
+      Big b = it->second;
+      big_free_.erase(it);
+      big_.push_back(b);
+      return (double *)b.base;
+    }
     bool pinned;
     char *p = raw(bytes, pinned);
     if (!p) fail(MICCO_ERR_OOM, "host allocation failed");
-    big_.push_back({p, pinned});
+    big_.push_back({p, bytes, pinned});
     return (double *)p;
   }
   while (cur_ < chunks_.size() && chunks_[cur_].used + bytes > chunks_[cur_].size) ++cur_;

@@ -10,6 +10,7 @@
 #include <cstring>
 #include <memory>
 #include <string>
+#include <map>
 #include <unordered_map>
 #include <vector>
 
@@ -123,7 +124,9 @@ class HostArena {
  private:
   struct Chunk { char *base; int64_t size, used; bool pinned; };
   std::vector<Chunk> chunks_;
-  std::vector<std::pair<char *, bool>> big_;
+  struct Big { char *base; int64_t size; bool pinned; };
+  std::vector<Big> big_;                  // blocks larger than a chunk, in use this round
+  std::multimap<int64_t, Big> big_free_;  // kept across rewind(), reused by size
   size_t cur_ = 0;  // chunk being filled
   bool pinned_ = true;
 };

@@ -558,14 +558,13 @@ constexpr int DOT_SMEM = 2 * 32 * 33 * 16;  // two 32×33 complex tiles (33.8 KB
 __device__ __forceinline__ void zdot_body(const DotDesc *__restrict__ descs, int n_desc) {
   extern __shared__ __align__(16) double2 dsm[];
   __shared__ double red[2][DT / 32];
+  // Slice-major CTA order (every task of the launch has Lt CTAs): the CTAs resident at any
+  // moment cover a few slices of every dot, so an operand shared by several dots of the launch
+  // (C4's c = 2 products are each read by ~70 dots) is read from DRAM once per slice and
+  // served from L2 afterwards; task-major order kept whole operands live and re-read them.
   const long long cta = blockIdx.x;
-  int lo = 0, hi = n_desc - 1;
-  while (lo < hi) {
-    int mid = (lo + hi + 1) >> 1;
-    if (descs[mid].cta_begin <= cta) lo = mid; else hi = mid - 1;
-  }
-  const DotDesc &d = descs[lo];
-  const int t = (int)(cta - d.cta_begin);
+  const int t = (int)(cta / n_desc);
+  const DotDesc &d = descs[cta - (long long)t * n_desc];
   const int tid = threadIdx.x;
   const double2 *A = d.A + t * d.sAt;
   const double2 *B = d.B ? d.B + t * d.sBt : nullptr;

@@ -52,7 +52,7 @@ struct DotDesc {
   int O[3], pad0;
   long long sAo[3], sBo[3];
   int Lt, pad1;
-  long long cta_begin;   // first CTA of this task in the grouped launch (one CTA per slice)
+  long long cta_begin;   // (unused by the kernel: CTA = t * n_desc + task, one per slice)
 };
 
 constexpr int kGemmBM = 64, kGemmBN = 64, kGemmBK = 8, kGemmStages = 4, kGemmThreads = 128;
