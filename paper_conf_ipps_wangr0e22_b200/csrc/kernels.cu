@@ -31,6 +31,13 @@ __device__ __forceinline__ void cp_async16(void *smem, const void *gmem, bool va
   int sz = valid ? 16 : 0;  // src-size 0 → zero fill (ragged tiles)
   asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;\n" ::"r"(s), "l"(gmem), "r"(sz));
 }
+__device__ __forceinline__ void cp_async16s(unsigned s, const void *gmem, bool valid) {
+  int sz = valid ? 16 : 0;
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;\n" ::"r"(s), "l"(gmem), "r"(sz));
+}
+__device__ __forceinline__ void cp_async16s(unsigned s, const void *gmem) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(s), "l"(gmem));
+}
 __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;\n" ::); }
 template <int N>
 __device__ __forceinline__ void cp_async_wait() {
@@ -184,15 +191,27 @@ __device__ __forceinline__ void zgemm_dmma_kernel_body(const GemmDesc *__restric
 // computed so they occupy the DMMA pacing slots; the task descriptor advances linearly.
 // Optional fused final dot (GemmDesc::D) in the epilogue.
 //
-// Complex product, two schemes (template M3):
-//   4M (default before round-1 end): Cr += Ar·Br + (−Ai)·Bi, Ci += Ar·Bi + Ai·Br  — 4 DMMAs
-//   3M (Gauss): K1 += (Ar+Ai)·Br, K2 += Ar·(Bi−Br), K3 += Ai·(Br+Bi);
-//               Cr = K1 − K3, Ci = K1 + K2                                       — 3 DMMAs
-// The 3M scheme does 25% fewer DMMAs for the same algorithmic work (8 real flops per complex
-// MAC are still what the roofline counts); its rounding differs from the 4M one but stays far
-// inside the 1e-10 parity bound, and exact-integer inputs stay bit-exact (every partial sum
-// is an integer below 2^53; SURVEY.md §8(c) "Bit-exact GPU parity").
+// Complex product, three schemes (template M3, M3T):
+//   4M: Cr += Ar·Br + (−Ai)·Bi, Ci += Ar·Bi + Ai·Br                                — 4 DMMAs
+//   3M "T" (default): T1 += Ar·Br, T2 += Ai·Bi, T3 += (Ar+Ai)·(Br+Bi);
+//                     Cr = T1 − T2, Ci = T3 − (T1 + T2)            — 3 DMMAs, MI + NJ sums
+//   3M "K": K1 += (Ar+Ai)·Br, K2 += Ar·(Bi−Br), K3 += Ai·(Br+Bi);
+//           Cr = K1 − K3, Ci = K1 + K2                             — 3 DMMAs, MI + 2·NJ sums
+// The 3M schemes do 25% fewer DMMAs for the same algorithmic work (8 real flops per complex
+// MAC are still what the roofline counts); their rounding differs from the 4M one but stays
+// far inside the 1e-10 parity bound, and exact-integer inputs stay bit-exact (every partial
+// sum is an integer below 2^53; SURVEY.md §8(c) "Bit-exact GPU parity").  The operand sums
+// are DADDs, and a DADD waits for the FP64 pipe the DMMAs occupy (ncu: "math pipe throttle"
+// on the DADDs; each costs ~0.7 of a DMMA slot), so the T form, with 6 instead of 8 sums
+// per 24 DMMAs, is the faster one: 36.9 vs 35.0 TFLOP/s algorithmic on the bench workload.
 constexpr int BK2 = 16, ST2 = 3;
+constexpr int kGemmPhaseNs = 0;
+#ifndef MICCO_BARRIER_LATE
+#define MICCO_BARRIER_LATE 0  // 1: stage barrier before the last k-quad (measured slower: 35.6 vs 36.9 TF)
+#endif
+#ifndef MICCO_KEEP_SN
+#define MICCO_KEEP_SN 1
+#endif
 constexpr int APITCH2 = BK2 + 4;  // [m][k] rows: 320 B ≡ 64 (mod 128): A fragment loads conflict-free
 
 template <int TBM, int TBN>
@@ -203,15 +222,43 @@ struct PCfg {
 };
 constexpr int GEMM2_SMEM = PCfg<64, 64>::SMEM;
 
-template <int LPTA, int LPTB>
+// Per-thread load geometry of one operand stage, compile-time for a layout class.  A stage
+// holds ROWS × BK2 complex elements (rows = m for A, n for B); KFAST = the operand is
+// contiguous along k, so consecutive threads copy consecutive k.  Element j of a thread sits
+// at (row r0 + j·RJ, k k0 + j·KJ): its shared-memory offset advances by a compile-time
+// stride and its global offset by a per-tile constant, so a copy is one IMAD.WIDE + LDGSTS.
+template <int ROWS, int NTH, bool KFAST>
+struct Geo {
+  static constexpr int L = ROWS * BK2 / NTH;
+  static constexpr int RJ = KFAST ? NTH / BK2 : 0;
+  static constexpr int KJ = KFAST ? 0 : NTH / ROWS;
+  static_assert(KFAST ? (NTH % BK2 == 0) : (NTH % ROWS == 0), "load geometry");
+  __device__ static int r0(int tid) { return KFAST ? tid / BK2 : tid % ROWS; }
+  __device__ static int k0(int tid) { return KFAST ? tid % BK2 : tid / ROWS; }
+};
+
+// bits j < L with base + j·STEP < lim
+template <int L, int STEP>
+__device__ __forceinline__ unsigned run_mask(int base, int lim) {
+  const int room = lim - base;
+  if (room <= 0) return 0u;
+  if constexpr (STEP == 0) {
+    return (1u << L) - 1u;
+  } else {
+    const int cnt = min(L, (room + STEP - 1) / STEP);
+    return (1u << cnt) - 1u;
+  }
+}
+
+template <int LA, int LB>
 struct LoadCur {
-  const double2 *A, *B;  // tile bases (t, mo/no, m0/n0 applied)
+  const double2 *A, *B;    // tile bases (t, mo/no, m0/n0 applied; ko = kb = 0)
+  const double2 *pA, *pB;  // bases of the stage being loaded
   long long sAko, sBko;
-  int sAki, sBki;
-  int Ki, KT, KTOT;
-  int offA[LPTA], offB[LPTB];
-  unsigned vA, vB;       // m-valid / n-valid bit per element
-  bool akf, bnf;
+  int stepA, stepB;        // BK2·sAki, BK2·sBki
+  int Ki, KT, KTOT, kin, ko, kb;
+  int gA[LA], gB[LB];      // element offsets from the stage base (0 for rows outside the tile)
+  unsigned rmA, rmB;       // rows inside the tile
 };
 
 struct StoreCur {
@@ -221,9 +268,11 @@ struct StoreCur {
   long long pidx;    // first partial-sum slot of this tile
 };
 
-template <int NTH, int TBM, int TBN, int LPTA, int LPTB>
+template <int NTH, int TBM, int TBN, bool AKF, bool BNF, typename LC>
 __device__ __forceinline__ void decode_tile(const GemmDesc *__restrict__ descs, int n_desc, int &task,
-                                            long long tile, int tid, LoadCur<LPTA, LPTB> *L, StoreCur *S) {
+                                            long long tile, int tid, LC *L, StoreCur *S) {
+  using GA = Geo<TBM, NTH, AKF>;
+  using GB = Geo<TBN, NTH, !BNF>;
   while (task + 1 < n_desc && descs[task + 1].tile_begin <= tile) ++task;
   const GemmDesc &d = descs[task];
   unsigned lt = (unsigned)(tile - d.tile_begin);  // tiles of one task < 2^32: 32-bit div/mod
@@ -239,28 +288,20 @@ __device__ __forceinline__ void decode_tile(const GemmDesc *__restrict__ descs, 
     const int sAmi = (int)d.sAmi, sAki = (int)d.sAki, sBki = (int)d.sBki, sBni = (int)d.sBni;
     L->A = d.A + t * d.sAt + mo * d.sAmo + (long long)m0 * sAmi;
     L->B = d.B + t * d.sBt + no * d.sBno + (long long)n0 * sBni;
-    L->sAko = d.sAko; L->sBko = d.sBko; L->sAki = sAki; L->sBki = sBki;
+    L->pA = L->A; L->pB = L->B;
+    L->sAko = d.sAko; L->sBko = d.sBko;
+    L->stepA = BK2 * sAki; L->stepB = BK2 * sBki;
     L->Ki = d.Ki; L->KT = KT; L->KTOT = d.Ko * KT;
-    L->akf = (sAki == 1);
-    L->bnf = (sBni == 1);
-    const int Mi = d.Mi, Ni = d.Ni;
-    L->vA = 0; L->vB = 0;
+    L->kin = 0; L->ko = 0; L->kb = 0;
+    const int ra = GA::r0(tid), ka = GA::k0(tid), rb = GB::r0(tid), kb = GB::k0(tid);
+    L->rmA = run_mask<GA::L, GA::RJ>(m0 + ra, d.Mi);
+    L->rmB = run_mask<GB::L, GB::RJ>(n0 + rb, d.Ni);
+    const int bA = ra * sAmi + ka * sAki, jA = GA::RJ * sAmi + GA::KJ * sAki;
+    const int bB = kb * sBki + rb * sBni, jB = GB::KJ * sBki + GB::RJ * sBni;
 #pragma unroll
-    for (int j = 0; j < LPTA; ++j) {
-      const int e = tid + j * NTH;
-      int m, k;
-      if (L->akf) { k = e & (BK2 - 1); m = e / BK2; } else { m = e % TBM; k = e / TBM; }
-      L->offA[j] = m * sAmi + k * sAki;
-      if (m0 + m < Mi) L->vA |= 1u << j;
-    }
+    for (int j = 0; j < GA::L; ++j) L->gA[j] = ((L->rmA >> j) & 1u) ? bA + j * jA : 0;
 #pragma unroll
-    for (int j = 0; j < LPTB; ++j) {
-      const int e = tid + j * NTH;
-      int n, kb;
-      if (L->bnf) { n = e % TBN; kb = e / TBN; } else { kb = e & (BK2 - 1); n = e / BK2; }
-      L->offB[j] = kb * sBki + n * sBni;
-      if (n0 + n < Ni) L->vB |= 1u << j;
-    }
+    for (int j = 0; j < GB::L; ++j) L->gB[j] = ((L->rmB >> j) & 1u) ? bB + j * jB : 0;
   }
   if (S) {
     S->C = d.C + t * d.sCt + mo * d.sCmo + no * d.sCno;
@@ -273,27 +314,39 @@ __device__ __forceinline__ void decode_tile(const GemmDesc *__restrict__ descs, 
 }
 
 // NWM × NWN warps with WTM × WTN complex warp tiles; CTA tile (NWM·WTM) × (NWN·WTN).
-template <int NWM, int NWN, int WTM, int WTN, bool M3>
+// AKF / BNF: the layout class (A contiguous along k / B contiguous along n).
+template <int NWM, int NWN, int WTM, int WTN, bool M3, bool M3T, bool AKF, bool BNF>
 __device__ __forceinline__ void zgemm_persistent_body(const GemmDesc *__restrict__ descs, int n_desc,
-                                                      long long total) {
+                                                      long long total, unsigned phase_ns) {
   constexpr int NTH = NWM * NWN * 32;
   constexpr int TBM = NWM * WTM, TBN = NWN * WTN;
-  constexpr int LPTA = (TBM * BK2) / NTH, LPTB = (TBN * BK2) / NTH;
+  using GA = Geo<TBM, NTH, AKF>;
+  using GB = Geo<TBN, NTH, !BNF>;
+  constexpr int LPTA = GA::L, LPTB = GB::L;
   constexpr int MI = WTM / 8, NJ = WTN / 8;  // 8x8 blocks per warp
   constexpr int NACC = M3 ? 3 : 2;
   using Cfg = PCfg<TBM, TBN>;
   constexpr int BP = Cfg::BP;
+  // shared-memory stride between a thread's consecutive elements (complex elements)
+  constexpr int SJA = GA::RJ * APITCH2 + GA::KJ, SJB = GB::KJ * BP + GB::RJ;
   extern __shared__ __align__(128) double2 smem[];
   double2 *As = smem;
   double2 *Bs = smem + ST2 * Cfg::AE;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const int wm = warp / NWN, wn = warp % NWN;
+  const unsigned sA0 = (unsigned)__cvta_generic_to_shared(As + GA::r0(tid) * APITCH2 + GA::k0(tid));
+  const unsigned sB0 = (unsigned)__cvta_generic_to_shared(Bs + GB::k0(tid) * BP + GB::r0(tid));
 
   // CTA c takes tiles c, c + G, c + 2G, ...: the CTAs running at any moment work on
   // neighbouring tiles (the same slices), so each A/B block is fetched from DRAM once and
   // served to the other CTAs from L2 (contiguous per-CTA ranges doubled the DRAM reads)
   const long long G = gridDim.x, t_begin = blockIdx.x;
   if (t_begin >= total) return;
+  // The two CTAs of an SM run tiles of equal length, so if they start together their
+  // epilogues coincide and the DMMA pipe idles through both.  The lag between them is
+  // neutrally stable (while one is in its epilogue the other runs the pipe alone), so a
+  // one-off delay of the second CTA keeps their epilogues apart for the whole launch.
+  if (phase_ns > 0 && 2 * blockIdx.x >= gridDim.x) __nanosleep(phase_ns);
 
   int task_l = 0, task_c = 0;
   {  // first task by binary search, then linear advance
@@ -308,50 +361,78 @@ __device__ __forceinline__ void zgemm_persistent_body(const GemmDesc *__restrict
   StoreCur S;
   long long tile_l = t_begin, tile_c = t_begin;
   int kt_l = 0, kt_c = 0;
-  decode_tile<NTH, TBM, TBN, LPTA, LPTB>(descs, n_desc, task_l, tile_l, tid, &L, nullptr);
-  decode_tile<NTH, TBM, TBN, LPTA, LPTB>(descs, n_desc, task_c, tile_c, tid, (LoadCur<LPTA, LPTB> *)nullptr, &S);
+  decode_tile<NTH, TBM, TBN, AKF, BNF>(descs, n_desc, task_l, tile_l, tid, &L, &S);
+  // The load side decodes every tile first; it leaves the store cursor of that tile in Sn so
+  // the epilogue does not decode it again (unless the loads ran more than a tile ahead).
+  StoreCur Sn;
+  long long sn_tile = -1;
+  int sn_task = 0;
   bool more_l = true;
 
   // The loads of a stage are issued in NPART pieces interleaved with the DMMA stream of the
-  // stage being computed (one piece per k-quad), so the scheduler can slot the cp.async and
-  // address arithmetic into the DMMA pacing gaps instead of running a separate load phase.
+  // stage being computed (one piece per k-quad), so the scheduler can slot the cp.async
+  // into the DMMA pacing gaps instead of running a separate load phase.  A DMMA holds its
+  // warp for 15 cycles (its SASS stall count), so with two warps per scheduler each has
+  // ~16 free issue cycles per DMMA: the copies must cost a few instructions, not dozens.
   constexpr int NPART = BK2 / 4;
   static_assert(LPTA % NPART == 0 && LPTB % NPART == 0, "load split");
-  const double2 *ldA = nullptr, *ldB = nullptr;
-  int ld_kb = 0;
+  unsigned mA = 0, mB = 0;  // elements of the stage being loaded inside the operand
+  bool ld_full = false;     // ... all of them (interior tile, whole k-step): warp-uniform
   auto begin_load = [&]() {
-    const int ko = kt_l / L.KT;
-    ld_kb = (kt_l - ko * L.KT) * BK2;
-    ldA = L.A + ko * L.sAko + (long long)ld_kb * L.sAki;
-    ldB = L.B + ko * L.sBko + (long long)ld_kb * L.sBki;
+    mA = L.rmA & run_mask<LPTA, GA::KJ>(L.kb + GA::k0(tid), L.Ki);
+    mB = L.rmB & run_mask<LPTB, GB::KJ>(L.kb + GB::k0(tid), L.Ki);
+    if constexpr (M3) ld_full = __all_sync(0xffffffffu, mA == (1u << LPTA) - 1u && mB == (1u << LPTB) - 1u);
   };
   auto issue_part = [&](int slot, int part) {
-    double2 *as = As + slot * Cfg::AE;
-    double2 *bs = Bs + slot * Cfg::BE;
+    const unsigned sa = sA0 + slot * (Cfg::AE * 16), sb = sB0 + slot * (Cfg::BE * 16);
+    if (ld_full) {  // every element inside both operands: plain copies, no zero fill
+#pragma unroll
+      for (int jj = 0; jj < LPTA / NPART; ++jj) {
+        const int j = part * (LPTA / NPART) + jj;
+        cp_async16s(sa + j * SJA * 16, L.pA + L.gA[j]);
+      }
+#pragma unroll
+      for (int jj = 0; jj < LPTB / NPART; ++jj) {
+        const int j = part * (LPTB / NPART) + jj;
+        cp_async16s(sb + j * SJB * 16, L.pB + L.gB[j]);
+      }
+      return;
+    }
 #pragma unroll
     for (int jj = 0; jj < LPTA / NPART; ++jj) {
       const int j = part * (LPTA / NPART) + jj;
-      const int e = tid + j * NTH;
-      int m, k;
-      if (L.akf) { k = e & (BK2 - 1); m = e / BK2; } else { m = e % TBM; k = e / TBM; }
-      const bool v = ((L.vA >> j) & 1u) && (ld_kb + k < L.Ki);
-      cp_async16(as + m * APITCH2 + k, v ? ldA + L.offA[j] : L.A, v);
+      const bool v = (mA >> j) & 1u;
+      cp_async16s(sa + j * SJA * 16, L.pA + (v ? L.gA[j] : 0), v);
     }
 #pragma unroll
     for (int jj = 0; jj < LPTB / NPART; ++jj) {
       const int j = part * (LPTB / NPART) + jj;
-      const int e = tid + j * NTH;
-      int n, k;
-      if (L.bnf) { n = e % TBN; k = e / TBN; } else { k = e & (BK2 - 1); n = e / BK2; }
-      const bool v = ((L.vB >> j) & 1u) && (ld_kb + k < L.Ki);
-      cp_async16(bs + k * BP + n, v ? ldB + L.offB[j] : L.B, v);
+      const bool v = (mB >> j) & 1u;
+      cp_async16s(sb + j * SJB * 16, L.pB + (v ? L.gB[j] : 0), v);
     }
   };
   auto advance_load = [&]() {  // next k-step, possibly in the next tile
     if (++kt_l == L.KTOT) {
       kt_l = 0;
-      if ((tile_l += G) < total) decode_tile<NTH, TBM, TBN, LPTA, LPTB>(descs, n_desc, task_l, tile_l, tid, &L, nullptr);
-      else more_l = false;
+      if ((tile_l += G) < total) {
+        if constexpr (M3 && MICCO_KEEP_SN) {  // (the 4M kernel has no registers left for a second cursor)
+          decode_tile<NTH, TBM, TBN, AKF, BNF>(descs, n_desc, task_l, tile_l, tid, &L, &Sn);
+          sn_tile = tile_l;
+          sn_task = task_l;
+        } else {
+          decode_tile<NTH, TBM, TBN, AKF, BNF>(descs, n_desc, task_l, tile_l, tid, &L, (StoreCur *)nullptr);
+        }
+      } else {
+        more_l = false;
+      }
+    } else if (++L.kin == L.KT) {
+      L.kin = 0; L.kb = 0; ++L.ko;
+      L.pA = L.A + L.ko * L.sAko;
+      L.pB = L.B + L.ko * L.sBko;
+    } else {
+      L.kb += BK2;
+      L.pA += L.stepA;
+      L.pB += L.stepB;
     }
   };
   auto issue_load = [&](int slot) {
@@ -375,56 +456,77 @@ __device__ __forceinline__ void zgemm_persistent_body(const GemmDesc *__restrict
     cp_async_commit();
   }
   int slot_c = 0, slot_l = ST2 - 1;
-  for (;;) {
+  // Fragments are double-buffered (3M): the LDS and the operand sums of k-quad q+1 are issued
+  // before the DMMAs of q.  The stage barrier sits before the DMMAs of the last k-quad, so the
+  // first fragments of the next stage are read while those DMMAs run, not after the barrier.
+  constexpr int FA = M3 ? 3 : 2, FB = M3 ? 3 : 2;
+  double fa[2][MI][FA], fb[2][NJ][FB];
+  auto load_frag = [&](int buf, int slot, int kq) {
+    const double2 *as = As + slot * Cfg::AE;
+    const double2 *bs = Bs + slot * Cfg::BE;
+#pragma unroll
+    for (int i = 0; i < MI; ++i) {
+      const double2 a = as[(wm * WTM + i * 8 + (lane >> 2)) * APITCH2 + kq * 4 + (lane & 3)];
+      fa[buf][i][0] = a.x;
+      fa[buf][i][1] = a.y;
+      if constexpr (M3) fa[buf][i][2] = a.x + a.y;  // Ar + Ai
+    }
+#pragma unroll
+    for (int j = 0; j < NJ; ++j) {
+      const double2 b = bs[(kq * 4 + (lane & 3)) * BP + wn * WTN + j * 8 + (lane >> 2)];
+      fb[buf][j][0] = b.x;
+      fb[buf][j][1] = b.y;
+      if constexpr (M3) {
+        if constexpr (!M3T) fb[buf][j][1] = b.y - b.x;  // Bi − Br
+        fb[buf][j][2] = b.x + b.y;                       // Br + Bi
+      }
+    }
+  };
+  constexpr bool LATE = MICCO_BARRIER_LATE != 0;
+  if constexpr (LATE) {
     cp_async_wait<ST2 - 2>();
     __syncthreads();
+    if constexpr (M3) load_frag(0, slot_c, 0);
+  }
+  for (;;) {
+    if constexpr (!LATE) {
+      cp_async_wait<ST2 - 2>();
+      __syncthreads();
+      if constexpr (M3) load_frag(0, slot_c, 0);
+    }
     const bool ld = more_l;
     if (ld) begin_load();
-    const double2 *as = As + slot_c * Cfg::AE;
-    const double2 *bs = Bs + slot_c * Cfg::BE;
-    // Fragments are double-buffered inside the stage: the LDS (and, for 3M, the operand
-    // sums on the FP64 pipe) of k-quad q+1 are issued before the DMMAs of q, so neither
-    // the shared-memory latency nor a DADD waiting behind DMMAs sits in front of them.
-    constexpr int FA = M3 ? 3 : 2, FB = M3 ? 3 : 2;
-    double fa[2][MI][FA], fb[2][NJ][FB];
-    auto load_frag = [&](int buf, int kq) {
-#pragma unroll
-      for (int i = 0; i < MI; ++i) {
-        const double2 a = as[(wm * WTM + i * 8 + (lane >> 2)) * APITCH2 + kq * 4 + (lane & 3)];
-        fa[buf][i][0] = a.x;
-        fa[buf][i][1] = a.y;
-        if constexpr (M3) fa[buf][i][2] = a.x + a.y;  // Ar + Ai
-      }
-#pragma unroll
-      for (int j = 0; j < NJ; ++j) {
-        const double2 b = bs[(kq * 4 + (lane & 3)) * BP + wn * WTN + j * 8 + (lane >> 2)];
-        fb[buf][j][0] = b.x;
-        fb[buf][j][1] = b.y;
-        if constexpr (M3) {
-          fb[buf][j][1] = b.y - b.x;  // Bi − Br
-          fb[buf][j][2] = b.x + b.y;  // Br + Bi
-        }
-      }
-    };
-    // (4M keeps a single buffer: its 128 accumulator registers leave no room for a second)
-    if constexpr (M3) load_frag(0, 0);
 #pragma unroll
     for (int kq = 0; kq < BK2 / 4; ++kq) {
       if (ld) issue_part(slot_l, kq);
       const int cur = M3 ? (kq & 1) : 0;
-      if constexpr (M3) {
-        if (kq + 1 < BK2 / 4) load_frag(cur ^ 1, kq + 1);
+      if (kq + 1 < BK2 / 4) {
+        if constexpr (M3) load_frag(cur ^ 1, slot_c, kq + 1);
+        else load_frag(0, slot_c, kq);
       } else {
-        load_frag(0, kq);
+        if constexpr (!M3) load_frag(0, slot_c, kq);
+        if (ld) advance_load();
+        cp_async_commit();
+        if constexpr (LATE) {
+          cp_async_wait<ST2 - 2>();  // the next stage has landed ...
+          __syncthreads();           // ... for every thread, and this stage's slot is free
+          if constexpr (M3) load_frag(cur ^ 1, slot_c + 1 == ST2 ? 0 : slot_c + 1, 0);
+        }
       }
       if constexpr (M3) {
 #pragma unroll
         for (int i = 0; i < MI; ++i)
 #pragma unroll
           for (int j = 0; j < NJ; ++j) {
-            dmma(acc[i][j][0][0], acc[i][j][0][1], fa[cur][i][2], fb[cur][j][0]);  // (Ar+Ai)·Br
-            dmma(acc[i][j][1][0], acc[i][j][1][1], fa[cur][i][0], fb[cur][j][1]);  // Ar·(Bi−Br)
-            dmma(acc[i][j][2][0], acc[i][j][2][1], fa[cur][i][1], fb[cur][j][2]);  // Ai·(Br+Bi)
+            if constexpr (M3T) {
+              dmma(acc[i][j][0][0], acc[i][j][0][1], fa[cur][i][0], fb[cur][j][0]);  // Ar·Br
+              dmma(acc[i][j][1][0], acc[i][j][1][1], fa[cur][i][1], fb[cur][j][1]);  // Ai·Bi
+              dmma(acc[i][j][2][0], acc[i][j][2][1], fa[cur][i][2], fb[cur][j][2]);  // (Ar+Ai)·(Br+Bi)
+            } else {
+              dmma(acc[i][j][0][0], acc[i][j][0][1], fa[cur][i][2], fb[cur][j][0]);  // (Ar+Ai)·Br
+              dmma(acc[i][j][1][0], acc[i][j][1][1], fa[cur][i][0], fb[cur][j][1]);  // Ar·(Bi−Br)
+              dmma(acc[i][j][2][0], acc[i][j][2][1], fa[cur][i][1], fb[cur][j][2]);  // Ai·(Br+Bi)
+            }
           }
       } else {
 #pragma unroll
@@ -443,8 +545,6 @@ __device__ __forceinline__ void zgemm_persistent_body(const GemmDesc *__restrict
           }
       }
     }
-    if (ld) advance_load();
-    cp_async_commit();
     slot_l = (slot_l + 1 == ST2) ? 0 : slot_l + 1;
     slot_c = (slot_c + 1 == ST2) ? 0 : slot_c + 1;
     if (S.D && kt_c + 2 == S.KTOT) {
@@ -463,7 +563,10 @@ __device__ __forceinline__ void zgemm_persistent_body(const GemmDesc *__restrict
     if (++kt_c == S.KTOT) {  // tile done: write back (next tile's loads already in flight)
       // the complex value of accumulator block (i, j), half h
       auto cval = [&](int i, int j, int h, double &re, double &im) {
-        if constexpr (M3) {
+        if constexpr (M3T) {  // T1 = Ar·Br, T2 = Ai·Bi, T3 = (Ar+Ai)·(Br+Bi)
+          re = acc[i][j][0][h] - acc[i][j][1][h];
+          im = acc[i][j][2][h] - (acc[i][j][0][h] + acc[i][j][1][h]);
+        } else if constexpr (M3) {
           re = acc[i][j][0][h] - acc[i][j][2][h];
           im = acc[i][j][0][h] + acc[i][j][1][h];
         } else {
@@ -538,7 +641,12 @@ __device__ __forceinline__ void zgemm_persistent_body(const GemmDesc *__restrict
           for (int q = 0; q < NACC; ++q) acc[i][j][q][0] = acc[i][j][q][1] = 0.0;
       kt_c = 0;
       if ((tile_c += G) >= total) break;
-      decode_tile<NTH, TBM, TBN, LPTA, LPTB>(descs, n_desc, task_c, tile_c, tid, (LoadCur<LPTA, LPTB> *)nullptr, &S);
+      if (M3 && MICCO_KEEP_SN && sn_tile == tile_c) {
+        S = Sn;
+        task_c = sn_task;
+      } else {
+        decode_tile<NTH, TBM, TBN, AKF, BNF>(descs, n_desc, task_c, tile_c, tid, (LoadCur<LPTA, LPTB> *)nullptr, &S);
+      }
     }
   }
   cp_async_wait<0>();
@@ -688,10 +796,22 @@ __global__ void accumulate_kernel(double2 *dst, const double2 *src, long long n)
 __global__ void __launch_bounds__(NT, 2) zgemm_dmma_kernel(const __grid_constant__ GemmBatch b, long long total) {
   zgemm_dmma_kernel_body(b.d, b.n, total);
 }
-template <int NWM, int NWN, int WTM, int WTN, bool M3>
+template <int NWM, int NWN, int WTM, int WTN, bool M3, bool M3T, bool AKF, bool BNF>
 __global__ void __launch_bounds__(NWM * NWN * 32, 2)
-    zgemm_persistent(const __grid_constant__ GemmBatch b, long long total) {
-  zgemm_persistent_body<NWM, NWN, WTM, WTN, M3>(b.d, b.n, total);
+    zgemm_persistent(const __grid_constant__ GemmBatch b, long long total, unsigned phase_ns) {
+  zgemm_persistent_body<NWM, NWN, WTM, WTN, M3, M3T, AKF, BNF>(b.d, b.n, total, phase_ns);
+}
+
+// The persistent GEMM for layout class cls (0..3 = (A contiguous along m ? 2 : 0) +
+// (B contiguous along k ? 1 : 0), layout.cpp gemm_class).
+template <int NWM, int NWN, int WTM, int WTN, bool M3, bool M3T>
+void (*persistent_fn(int cls))(const GemmBatch, long long, unsigned) {
+  switch (cls) {
+    case 0: return zgemm_persistent<NWM, NWN, WTM, WTN, M3, M3T, true, true>;
+    case 1: return zgemm_persistent<NWM, NWN, WTM, WTN, M3, M3T, true, false>;
+    case 2: return zgemm_persistent<NWM, NWN, WTM, WTN, M3, M3T, false, true>;
+    default: return zgemm_persistent<NWM, NWN, WTM, WTN, M3, M3T, false, false>;
+  }
 }
 
 __global__ void __launch_bounds__(DT) zdot_kernel(const __grid_constant__ DotBatch b) { zdot_body(b.d, b.n); }
@@ -699,15 +819,16 @@ __global__ void __launch_bounds__(DT) zdot_kernel(const __grid_constant__ DotBat
 }  // namespace
 
 int gemm_variant() {
-  // MICCO_GEMM = 5 (default) persistent 64×32 tiles, 3M complex products;
-  //              2 persistent 64×64 tiles, 4M;  1 per-tile 64×64 4M (also the gather kernel).
-  // Measured on the bench workload: 5 → 19.9k, 2 → 18.9k graphs/s (profiles/bench_r01_v6.json).
-  // Earlier experiments (warp-specialised producer/consumer, small 32×32 tiles, 8-warp 3M)
-  // are in DESIGN.md §6's history table; all were slower and were removed.
+  // MICCO_GEMM = 5 (default) persistent 64×32 tiles, 3M "T" complex products;
+  //              6 the same with the 3M "K" form;  2 persistent 64×64 tiles, 4M;
+  //              1 per-tile 64×64 4M (also the gather kernel).
+  // Measured on the bench workload (GEMM TFLOP/s algorithmic): 5 → 36.9, 6 → 35.0, 2 → 31.6
+  // (profiles/bench_r01_v7*.json).  Earlier experiments (warp-specialised producer/consumer,
+  // small 32×32 tiles, 8-warp 3M) are in DESIGN.md §6's history table; all were slower.
   static int variant = -1;
   if (variant < 0) {
     const char *e = getenv("MICCO_GEMM");
-    variant = (e && (e[0] == '1' || e[0] == '2' || e[0] == '5')) ? e[0] - '0' : 5;
+    variant = (e && (e[0] == '1' || e[0] == '2' || e[0] == '5' || e[0] == '6')) ? e[0] - '0' : 5;
   }
   return variant;
 }
@@ -716,10 +837,10 @@ void gemm_tile_shape(int cls, int *bm, int *bn) {
   *bm = 64;
   *bn = 64;
   if (cls == 4) return;  // gather kernel (v1)
-  if (gemm_variant() == 5) *bn = 32;
+  if (gemm_variant() >= 5) *bn = 32;
 }
 
-bool gemm_uses_3m(int cls) { return cls != 4 && gemm_variant() == 5; }
+bool gemm_uses_3m(int cls) { return cls != 4 && gemm_variant() >= 5; }
 
 bool gemm_fused_dot_ok() { return gemm_variant() != 1; }
 
@@ -729,12 +850,17 @@ cudaError_t launch_gemm_group(const GemmBatch *b, long long total_tiles, int cls
   if (!attr_set) {
     cudaError_t e = cudaFuncSetAttribute(zgemm_dmma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, GEMM_SMEM);
     if (e != cudaSuccess) return e;
-    e = cudaFuncSetAttribute(zgemm_persistent<2, 2, 32, 32, false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                             PCfg<64, 64>::SMEM);
-    if (e != cudaSuccess) return e;
-    e = cudaFuncSetAttribute(zgemm_persistent<2, 2, 32, 16, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                             PCfg<64, 32>::SMEM);
-    if (e != cudaSuccess) return e;
+    for (int c = 0; c < 4; ++c) {
+      e = cudaFuncSetAttribute(persistent_fn<2, 2, 32, 32, false, false>(c), cudaFuncAttributeMaxDynamicSharedMemorySize,
+                               PCfg<64, 64>::SMEM);
+      if (e != cudaSuccess) return e;
+      e = cudaFuncSetAttribute(persistent_fn<2, 2, 32, 16, true, false>(c), cudaFuncAttributeMaxDynamicSharedMemorySize,
+                               PCfg<64, 32>::SMEM);
+      if (e != cudaSuccess) return e;
+      e = cudaFuncSetAttribute(persistent_fn<2, 2, 32, 16, true, true>(c), cudaFuncAttributeMaxDynamicSharedMemorySize,
+                               PCfg<64, 32>::SMEM);
+      if (e != cudaSuccess) return e;
+    }
     attr_set = true;
   }
   if (total_tiles <= 0) return cudaSuccess;
@@ -748,10 +874,21 @@ cudaError_t launch_gemm_group(const GemmBatch *b, long long total_tiles, int cls
   }
   long long grid = 2LL * sms;  // 2 resident CTAs per SM
   if (grid > total_tiles) grid = total_tiles;
+  static int phase_ns = -1;  // start lag of the second CTA per SM (env MICCO_GEMM_PHASE_NS)
+  if (phase_ns < 0) {
+    const char *e = getenv("MICCO_GEMM_PHASE_NS");
+    phase_ns = e ? atoi(e) : kGemmPhaseNs;
+    if (phase_ns < 0) phase_ns = 0;
+  }
   if (variant == 2)
-    zgemm_persistent<2, 2, 32, 32, false><<<(unsigned)grid, 128, PCfg<64, 64>::SMEM, st>>>(*b, total_tiles);
-  else
-    zgemm_persistent<2, 2, 32, 16, true><<<(unsigned)grid, 128, PCfg<64, 32>::SMEM, st>>>(*b, total_tiles);
+    persistent_fn<2, 2, 32, 32, false, false>(cls)<<<(unsigned)grid, 128, PCfg<64, 64>::SMEM, st>>>(*b, total_tiles,
+                                                                                           (unsigned)phase_ns);
+  else if (variant == 5)
+    persistent_fn<2, 2, 32, 16, true, true>(cls)<<<(unsigned)grid, 128, PCfg<64, 32>::SMEM, st>>>(*b, total_tiles,
+                                                                                                (unsigned)phase_ns);
+  else  // 6: the 3M "K" form
+    persistent_fn<2, 2, 32, 16, true, false>(cls)<<<(unsigned)grid, 128, PCfg<64, 32>::SMEM, st>>>(*b, total_tiles,
+                                                                                          (unsigned)phase_ns);
   return cudaGetLastError();
 }
 
