@@ -349,7 +349,7 @@ struct Executor::Impl {
       Timed tm{devs[l.dev].timing_events.get(), devs[l.dev].timing_events.get(), kind, l.dev};
       CK(cudaEventRecord(tm.a, l.st));
       if constexpr (std::is_same<D, GemmDesc>::value) CK(launch_gemm_group(&b, total, cls, l.st));
-      else CK(launch_dot_group(&b, total, l.st));
+      else CK(launch_dot_group(&b, total, cls, l.st));
       CK(cudaEventRecord(tm.b, l.st));
       timed.push_back(tm);
       ++launches;
@@ -373,14 +373,21 @@ struct Executor::Impl {
           return acc;
         });
     }
-    launch_batch(l, l.dot, 1, 0, *dot_batch, kDotBatch, [](DotDesc *d, int cnt) {
-      long long acc = 0;
-      for (int i = 0; i < cnt; ++i) {
-        d[i].cta_begin = acc;
-        acc += d[i].Lt;
+    if (!l.dot.empty()) {  // one launch group per dot kernel (kernels.h dot_class)
+      std::vector<DotDesc> by[2];
+      for (const DotDesc &d : l.dot) by[dot_class(d.mode)].push_back(d);
+      l.dot.clear();
+      for (int c = 0; c < 2; ++c) {
+        launch_batch(l, by[c], 1, c, *dot_batch, kDotBatch, [](DotDesc *d, int cnt) {
+          long long acc = 0;
+          for (int i = 0; i < cnt; ++i) {
+            d[i].cta_begin = acc;
+            acc += d[i].Lt;
+          }
+          return acc;
+        });
       }
-      return acc;
-    });
+    }
     for (double2 *p : l.part_allocs) CK(cudaFreeAsync(p, l.st));
     l.part_allocs.clear();
   }
@@ -462,6 +469,8 @@ struct Executor::Impl {
         ok = dot_layout(A.rank, A.dim, B.rank, B.dim, tk.c, tk.pa, tk.pb, L);
       }
       if (!ok) fail(MICCO_ERR_UNSUPPORTED, "executor: dot layout");
+      if (L.sliceA > (1LL << 31) - 1)  // the dot kernel's short-run path indexes a slice in 32 bits
+        fail(MICCO_ERR_UNSUPPORTED, "executor: tensor slice exceeds 2^31 elements");
       DotDesc d{};
       d.A = pa; d.B = pb;
       d.out = devs[l.dev].scalars + (size_t)c.tensors[tk.out].scalar_slot * c.Lt;

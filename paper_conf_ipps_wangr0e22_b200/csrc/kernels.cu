@@ -679,19 +679,7 @@ __device__ __forceinline__ void zdot_body(const DotDesc *__restrict__ descs, int
   double sr = 0.0, si = 0.0;
   const long long O0 = d.O[0], O1 = d.O[1], O2 = d.O[2];
   const long long Ototal = O0 * O1 * O2;
-  if (d.mode == 3) {
-    for (int i = tid; i < d.X; i += DT) {
-      const double2 a = A[i];
-      sr += a.x;
-      si += a.y;
-    }
-  } else if (d.mode == 2) {
-    for (int i = tid; i < d.X; i += DT) {
-      const double2 a = A[(long long)i * d.sAx];
-      sr += a.x;
-      si += a.y;
-    }
-  } else if (d.mode == 0) {
+  if (d.mode == 0) {  // flat (outer, x) index, one element pair per thread per step
     const long long X = d.X, total = Ototal * X;
 #pragma unroll 4
     for (long long e = tid; e < total; e += DT) {
@@ -701,7 +689,7 @@ __device__ __forceinline__ void zdot_body(const DotDesc *__restrict__ descs, int
       const long long offB = o0 * d.sBo[0] + o1 * d.sBo[1] + o2 * d.sBo[2] + x * d.sBx;
       cmac(sr, si, A[offA], B[offB]);
     }
-  } else {  // transpose tiles: A contiguous along x, B contiguous along y (32×32 smem tiles)
+  } else {  // mode 1: A contiguous along x, B along y (32×32 shared-memory transpose tiles)
     double2 (*As)[33] = reinterpret_cast<double2 (*)[33]>(dsm);
     double2 (*Bs)[33] = reinterpret_cast<double2 (*)[33]>(dsm + 32 * 33);
     const int ty = tid >> 5, tx = tid & 31;
@@ -736,6 +724,41 @@ __device__ __forceinline__ void zdot_body(const DotDesc *__restrict__ descs, int
     for (int w = 0; w < DT / 32; ++w) { ar += red[0][w]; ai += red[1][w]; }
     d.out[t] = make_double2(ar, ai);
   }
+}
+
+// One warp per (dot, slice) for the short reductions (2: meson trace, 3: sum of the fused
+// GEMM's partials): no block barrier, a fixed-order butterfly (deterministic).  The flat
+// dots (mode 0) stay on the CTA kernel: a warp per C4 64×64 dot put 8× more slices in
+// flight, the working set outgrew L2 and the dots took 177 instead of 83 ms per step.
+constexpr int DW = DT / 32;  // items per CTA
+
+__device__ __forceinline__ void zdot_warp_body(const DotDesc *__restrict__ descs, int n_desc, long long items) {
+  const long long item = (long long)blockIdx.x * DW + (threadIdx.x >> 5);
+  if (item >= items) return;
+  const int t = (int)(item / n_desc);
+  const DotDesc &d = descs[item - (long long)t * n_desc];
+  const int lane = threadIdx.x & 31;
+  const double2 *A = d.A + t * d.sAt;
+  double sr = 0.0, si = 0.0;
+  if (d.mode == 3) {
+    for (int i = lane; i < d.X; i += 32) {
+      const double2 a = A[i];
+      sr += a.x;
+      si += a.y;
+    }
+  } else {  // mode 2
+    for (int i = lane; i < d.X; i += 32) {
+      const double2 a = A[(long long)i * d.sAx];
+      sr += a.x;
+      si += a.y;
+    }
+  }
+#pragma unroll
+  for (int off = 16; off > 0; off >>= 1) {
+    sr += __shfl_xor_sync(0xffffffffu, sr, off);
+    si += __shfl_xor_sync(0xffffffffu, si, off);
+  }
+  if (lane == 0) d.out[t] = make_double2(sr, si);
 }
 
 // ---------------------------------------------------------------- finalize / sum
@@ -815,6 +838,9 @@ void (*persistent_fn(int cls))(const GemmBatch, long long, unsigned) {
 }
 
 __global__ void __launch_bounds__(DT) zdot_kernel(const __grid_constant__ DotBatch b) { zdot_body(b.d, b.n); }
+__global__ void __launch_bounds__(DT) zdot_warp_kernel(const __grid_constant__ DotBatch b, long long items) {
+  zdot_warp_body(b.d, b.n, items);
+}
 
 }  // namespace
 
@@ -892,8 +918,12 @@ cudaError_t launch_gemm_group(const GemmBatch *b, long long total_tiles, int cls
   return cudaGetLastError();
 }
 
-cudaError_t launch_dot_group(const DotBatch *b, long long total_ctas, cudaStream_t st) {
+cudaError_t launch_dot_group(const DotBatch *b, long long total_ctas, int cls, cudaStream_t st) {
   if (total_ctas <= 0) return cudaSuccess;
+  if (cls == 0) {  // modes 2, 3: a warp per (dot, slice)
+    zdot_warp_kernel<<<(unsigned)((total_ctas + DW - 1) / DW), DT, 0, st>>>(*b, total_ctas);
+    return cudaGetLastError();
+  }
   static bool attr = false;
   if (!attr) {
     cudaError_t e = cudaFuncSetAttribute(zdot_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, DOT_SMEM);

@@ -83,7 +83,10 @@ bool gemm_fused_dot_ok();    // the selected persistent GEMM has the fused-dot e
 
 // Grouped launches: descs in device memory (all of one layout class); grid covers the tiles.
 cudaError_t launch_gemm_group(const GemmBatch *b, long long total_tiles, int cls, cudaStream_t st);
-cudaError_t launch_dot_group(const DotBatch *b, long long total_ctas, cudaStream_t st);
+// cls 0: a warp per dot and slice (modes 2, 3); cls 1: a CTA per dot and slice (modes 0, 1).
+// total_ctas = Σ Lt over the batch (one work item per dot and slice).
+inline int dot_class(int mode) { return mode == 0 || mode == 1 ? 1 : 0; }
+cudaError_t launch_dot_group(const DotBatch *b, long long total_ctas, int cls, cudaStream_t st);
 
 // vals[g][t] = Π_{c in comps(g)} S[slot_c][t] (component scalars)
 cudaError_t launch_finalize(int G, int Lt, const int *comp_off, const int *comp_slot,
