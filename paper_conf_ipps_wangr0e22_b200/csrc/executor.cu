@@ -418,7 +418,7 @@ struct Executor::Impl {
       d.sBko = L.sBko; d.sBki = L.sBki; d.sBno = L.sBno; d.sBni = L.sBni;
       d.sCmo = L.sCmo; d.sCmi = L.sCmi; d.sCno = L.sCno; d.sCni = L.sCni;
       d.Lt = c.Lt;
-      d.cls = gemm_class(L);
+      d.cls = gemm_kernel_class(gemm_class(L), L.Ko);
       int tbm, tbn;
       gemm_tile_shape(d.cls, &tbm, &tbn);
       d.tilesM = (L.Mi + tbm - 1) / tbm;

@@ -252,6 +252,7 @@ __device__ __forceinline__ unsigned run_mask(int base, int lim) {
 
 template <int LA, int LB>
 struct LoadCur {
+  static constexpr int NA = LA, NB = LB;
   const double2 *A, *B;    // tile bases (t, mo/no, m0/n0 applied; ko = kb = 0)
   const double2 *pA, *pB;  // bases of the stage being loaded
   long long sAko, sBko;
@@ -259,7 +260,26 @@ struct LoadCur {
   int Ki, KT, KTOT, kin, ko, kb;
   int gA[LA], gB[LB];      // element offsets from the stage base (0 for rows outside the tile)
   unsigned rmA, rmB;       // rows inside the tile
+  // blocked-K geometry (class kGemmClassKB): a stage is 4 ko × 4 ki, local k = 4·dko + dki;
+  // element j of a thread has local k kl0 + j·kls, shared offset s0 + j·sj (bytes)
+  int sAki, sBki, Ko, ko0, ki0;
+  int klA0, klAs, klB0, klBs;
+  unsigned sa0, sb0, sja, sjb;
 };
+
+// Per-thread blocked-K geometry of one operand (rows = m for A, n for B): the copy order
+// follows the operand's unit-stride index (ko, ki or the row), so warps read 64-byte runs.
+template <int ROWS, int NTH>
+__device__ __forceinline__ void kb_geo(int tid, long long sRow, long long sKo, long long sKi, int &r0, int &rj,
+                                       int &kl0, int &kls) {
+  if (sRow == 1 && sKo != 1 && sKi != 1) {  // row-fast
+    r0 = tid % ROWS; rj = 0; kl0 = tid / ROWS; kls = NTH / ROWS;
+  } else if (sKo == 1) {                     // ko-fast: dko = tid & 3, dki = (tid >> 2) & 3
+    r0 = tid / BK2; rj = NTH / BK2; kl0 = (tid & 3) * 4 + ((tid >> 2) & 3); kls = 0;
+  } else {                                   // ki-fast (also the gather fallback)
+    r0 = tid / BK2; rj = NTH / BK2; kl0 = tid & (BK2 - 1); kls = 0;
+  }
+}
 
 struct StoreCur {
   double2 *C;
@@ -268,7 +288,7 @@ struct StoreCur {
   long long pidx;    // first partial-sum slot of this tile
 };
 
-template <int NTH, int TBM, int TBN, bool AKF, bool BNF, typename LC>
+template <int NTH, int TBM, int TBN, bool AKF, bool BNF, bool KB, typename LC>
 __device__ __forceinline__ void decode_tile(const GemmDesc *__restrict__ descs, int n_desc, int &task,
                                             long long tile, int tid, LC *L, StoreCur *S) {
   using GA = Geo<TBM, NTH, AKF>;
@@ -283,8 +303,39 @@ __device__ __forceinline__ void decode_tile(const GemmDesc *__restrict__ descs, 
   const int mo = (int)(lt % Mo);
   const long long t = lt / Mo;
   const int m0 = tm * TBM, n0 = tn * TBN;
-  const int KT = (d.Ki + BK2 - 1) / BK2;
-  if (L) {
+  const int KT = KB ? ((d.Ko + 3) / 4) * ((d.Ki + 3) / 4) : (d.Ki + BK2 - 1) / BK2;
+  if (KB && L) {
+    const int sAmi = (int)d.sAmi, sBni = (int)d.sBni;
+    L->A = d.A + t * d.sAt + mo * d.sAmo + (long long)m0 * sAmi;
+    L->B = d.B + t * d.sBt + no * d.sBno + (long long)n0 * sBni;
+    L->pA = L->A; L->pB = L->B;
+    L->sAko = d.sAko; L->sBko = d.sBko;
+    L->sAki = (int)d.sAki; L->sBki = (int)d.sBki;
+    L->Ki = d.Ki; L->Ko = d.Ko; L->KT = KT; L->KTOT = KT;
+    L->ko0 = 0; L->ki0 = 0;
+    int ra, rja, rb, rjb;
+    kb_geo<TBM, NTH>(tid, d.sAmi, d.sAko, d.sAki, ra, rja, L->klA0, L->klAs);
+    kb_geo<TBN, NTH>(tid, d.sBni, d.sBko, d.sBki, rb, rjb, L->klB0, L->klBs);
+    L->sa0 = (unsigned)((ra * APITCH2 + L->klA0) * 16);
+    L->sja = (unsigned)((rja * APITCH2 + L->klAs) * 16);
+    L->sb0 = (unsigned)((L->klB0 * PCfg<TBM, TBN>::BP + rb) * 16);
+    L->sjb = (unsigned)((L->klBs * PCfg<TBM, TBN>::BP + rjb) * 16);
+    L->rmA = L->rmB = 0;
+#pragma unroll
+    for (int j = 0; j < LC::NA; ++j) {
+      const int m = ra + j * rja, kl = L->klA0 + j * L->klAs;
+      const bool v = m0 + m < d.Mi;
+      if (v) L->rmA |= 1u << j;
+      L->gA[j] = v ? (int)(m * d.sAmi + (kl >> 2) * d.sAko + (kl & 3) * d.sAki) : 0;
+    }
+#pragma unroll
+    for (int j = 0; j < LC::NB; ++j) {
+      const int n = rb + j * rjb, kl = L->klB0 + j * L->klBs;
+      const bool v = n0 + n < d.Ni;
+      if (v) L->rmB |= 1u << j;
+      L->gB[j] = v ? (int)(n * d.sBni + (kl >> 2) * d.sBko + (kl & 3) * d.sBki) : 0;
+    }
+  } else if (L) {
     const int sAmi = (int)d.sAmi, sAki = (int)d.sAki, sBki = (int)d.sBki, sBni = (int)d.sBni;
     L->A = d.A + t * d.sAt + mo * d.sAmo + (long long)m0 * sAmi;
     L->B = d.B + t * d.sBt + no * d.sBno + (long long)n0 * sBni;
@@ -307,7 +358,7 @@ __device__ __forceinline__ void decode_tile(const GemmDesc *__restrict__ descs, 
     S->C = d.C + t * d.sCt + mo * d.sCmo + no * d.sCno;
     S->sCmi = (int)d.sCmi; S->sCni = (int)d.sCni;
     S->Mi = d.Mi; S->Ni = d.Ni; S->m0 = m0; S->n0 = n0;
-    S->KTOT = d.Ko * KT;
+    S->KTOT = KB ? KT : d.Ko * KT;
     S->D = d.D ? d.D + t * d.sDt + mo * d.sDmo + no * d.sDno : nullptr;
     S->pidx = (tile - d.tile_begin) * (NTH / 32);
   }
@@ -315,12 +366,12 @@ __device__ __forceinline__ void decode_tile(const GemmDesc *__restrict__ descs, 
 
 // NWM × NWN warps with WTM × WTN complex warp tiles; CTA tile (NWM·WTM) × (NWN·WTN).
 // AKF / BNF: the layout class (A contiguous along k / B contiguous along n).
-template <int NWM, int NWN, int WTM, int WTN, bool M3, bool M3T, bool AKF, bool BNF>
+template <int NWM, int NWN, int WTM, int WTN, bool M3, bool M3T, bool AKF, bool BNF, bool KB = false>
 __device__ __forceinline__ void zgemm_persistent_body(const GemmDesc *__restrict__ descs, int n_desc,
                                                       long long total, unsigned phase_ns) {
   constexpr int NTH = NWM * NWN * 32;
   constexpr int TBM = NWM * WTM, TBN = NWN * WTN;
-  using GA = Geo<TBM, NTH, AKF>;
+  using GA = Geo<TBM, NTH, AKF>;  // (KB: only the element counts are used)
   using GB = Geo<TBN, NTH, !BNF>;
   constexpr int LPTA = GA::L, LPTB = GB::L;
   constexpr int MI = WTM / 8, NJ = WTN / 8;  // 8x8 blocks per warp
@@ -336,6 +387,7 @@ __device__ __forceinline__ void zgemm_persistent_body(const GemmDesc *__restrict
   const int wm = warp / NWN, wn = warp % NWN;
   const unsigned sA0 = (unsigned)__cvta_generic_to_shared(As + GA::r0(tid) * APITCH2 + GA::k0(tid));
   const unsigned sB0 = (unsigned)__cvta_generic_to_shared(Bs + GB::k0(tid) * BP + GB::r0(tid));
+  const unsigned sAs = (unsigned)__cvta_generic_to_shared(As), sBs = (unsigned)__cvta_generic_to_shared(Bs);
 
   // CTA c takes tiles c, c + G, c + 2G, ...: the CTAs running at any moment work on
   // neighbouring tiles (the same slices), so each A/B block is fetched from DRAM once and
@@ -361,7 +413,7 @@ __device__ __forceinline__ void zgemm_persistent_body(const GemmDesc *__restrict
   StoreCur S;
   long long tile_l = t_begin, tile_c = t_begin;
   int kt_l = 0, kt_c = 0;
-  decode_tile<NTH, TBM, TBN, AKF, BNF>(descs, n_desc, task_l, tile_l, tid, &L, &S);
+  decode_tile<NTH, TBM, TBN, AKF, BNF, KB>(descs, n_desc, task_l, tile_l, tid, &L, &S);
   // The load side decodes every tile first; it leaves the store cursor of that tile in Sn so
   // the epilogue does not decode it again (unless the loads ran more than a tile ahead).
   StoreCur Sn;
@@ -379,11 +431,48 @@ __device__ __forceinline__ void zgemm_persistent_body(const GemmDesc *__restrict
   unsigned mA = 0, mB = 0;  // elements of the stage being loaded inside the operand
   bool ld_full = false;     // ... all of them (interior tile, whole k-step): warp-uniform
   auto begin_load = [&]() {
-    mA = L.rmA & run_mask<LPTA, GA::KJ>(L.kb + GA::k0(tid), L.Ki);
-    mB = L.rmB & run_mask<LPTB, GB::KJ>(L.kb + GB::k0(tid), L.Ki);
-    if constexpr (M3) ld_full = __all_sync(0xffffffffu, mA == (1u << LPTA) - 1u && mB == (1u << LPTB) - 1u);
+    if constexpr (KB) {
+      if (L.ko0 + 4 <= L.Ko && L.ki0 + 4 <= L.Ki) {
+        mA = L.rmA;
+        mB = L.rmB;
+      } else {
+        unsigned ka = 0, kb = 0;
+#pragma unroll
+        for (int j = 0; j < LPTA; ++j) {
+          const int kl = L.klA0 + j * L.klAs;
+          if (L.ko0 + (kl >> 2) < L.Ko && L.ki0 + (kl & 3) < L.Ki) ka |= 1u << j;
+        }
+#pragma unroll
+        for (int j = 0; j < LPTB; ++j) {
+          const int kl = L.klB0 + j * L.klBs;
+          if (L.ko0 + (kl >> 2) < L.Ko && L.ki0 + (kl & 3) < L.Ki) kb |= 1u << j;
+        }
+        mA = L.rmA & ka;
+        mB = L.rmB & kb;
+      }
+    } else {
+      mA = L.rmA & run_mask<LPTA, GA::KJ>(L.kb + GA::k0(tid), L.Ki);
+      mB = L.rmB & run_mask<LPTB, GB::KJ>(L.kb + GB::k0(tid), L.Ki);
+    }
+    if constexpr (M3 && !KB) ld_full = __all_sync(0xffffffffu, mA == (1u << LPTA) - 1u && mB == (1u << LPTB) - 1u);
   };
   auto issue_part = [&](int slot, int part) {
+    if constexpr (KB) {  // runtime geometry (per task): element j at s0 + j·sj
+      const unsigned sa = sAs + slot * (Cfg::AE * 16) + L.sa0, sb = sBs + slot * (Cfg::BE * 16) + L.sb0;
+#pragma unroll
+      for (int jj = 0; jj < LPTA / NPART; ++jj) {
+        const int j = part * (LPTA / NPART) + jj;
+        const bool v = (mA >> j) & 1u;
+        cp_async16s(sa + j * L.sja, L.pA + (v ? L.gA[j] : 0), v);
+      }
+#pragma unroll
+      for (int jj = 0; jj < LPTB / NPART; ++jj) {
+        const int j = part * (LPTB / NPART) + jj;
+        const bool v = (mB >> j) & 1u;
+        cp_async16s(sb + j * L.sjb, L.pB + (v ? L.gB[j] : 0), v);
+      }
+      return;
+    }
     const unsigned sa = sA0 + slot * (Cfg::AE * 16), sb = sB0 + slot * (Cfg::BE * 16);
     if (ld_full) {  // every element inside both operands: plain copies, no zero fill
 #pragma unroll
@@ -416,15 +505,22 @@ __device__ __forceinline__ void zgemm_persistent_body(const GemmDesc *__restrict
       kt_l = 0;
       if ((tile_l += G) < total) {
         if constexpr (M3 && MICCO_KEEP_SN) {  // (the 4M kernel has no registers left for a second cursor)
-          decode_tile<NTH, TBM, TBN, AKF, BNF>(descs, n_desc, task_l, tile_l, tid, &L, &Sn);
+          decode_tile<NTH, TBM, TBN, AKF, BNF, KB>(descs, n_desc, task_l, tile_l, tid, &L, &Sn);
           sn_tile = tile_l;
           sn_task = task_l;
         } else {
-          decode_tile<NTH, TBM, TBN, AKF, BNF>(descs, n_desc, task_l, tile_l, tid, &L, (StoreCur *)nullptr);
+          decode_tile<NTH, TBM, TBN, AKF, BNF, KB>(descs, n_desc, task_l, tile_l, tid, &L, (StoreCur *)nullptr);
         }
       } else {
         more_l = false;
       }
+    } else if constexpr (KB) {
+      if ((L.ki0 += 4) >= L.Ki) {
+        L.ki0 = 0;
+        L.ko0 += 4;
+      }
+      L.pA = L.A + L.ko0 * L.sAko + L.ki0 * L.sAki;
+      L.pB = L.B + L.ko0 * L.sBko + L.ki0 * L.sBki;
     } else if (++L.kin == L.KT) {
       L.kin = 0; L.kb = 0; ++L.ko;
       L.pA = L.A + L.ko * L.sAko;
@@ -645,7 +741,7 @@ __device__ __forceinline__ void zgemm_persistent_body(const GemmDesc *__restrict
         S = Sn;
         task_c = sn_task;
       } else {
-        decode_tile<NTH, TBM, TBN, AKF, BNF>(descs, n_desc, task_c, tile_c, tid, (LoadCur<LPTA, LPTB> *)nullptr, &S);
+        decode_tile<NTH, TBM, TBN, AKF, BNF, KB>(descs, n_desc, task_c, tile_c, tid, (LoadCur<LPTA, LPTB> *)nullptr, &S);
       }
     }
   }
@@ -825,6 +921,12 @@ __global__ void __launch_bounds__(NWM * NWN * 32, 2)
   zgemm_persistent_body<NWM, NWN, WTM, WTN, M3, M3T, AKF, BNF>(b.d, b.n, total, phase_ns);
 }
 
+template <int NWM, int NWN, int WTM, int WTN, bool M3, bool M3T>
+__global__ void __launch_bounds__(NWM * NWN * 32, 2)
+    zgemm_persistent_kb(const __grid_constant__ GemmBatch b, long long total, unsigned phase_ns) {
+  zgemm_persistent_body<NWM, NWN, WTM, WTN, M3, M3T, true, true, true>(b.d, b.n, total, phase_ns);
+}
+
 // The persistent GEMM for layout class cls (0..3 = (A contiguous along m ? 2 : 0) +
 // (B contiguous along k ? 1 : 0), layout.cpp gemm_class).
 template <int NWM, int NWN, int WTM, int WTN, bool M3, bool M3T>
@@ -868,6 +970,14 @@ void gemm_tile_shape(int cls, int *bm, int *bn) {
 
 bool gemm_uses_3m(int cls) { return cls != 4 && gemm_variant() >= 5; }
 
+int gemm_kernel_class(int layout_cls, int Ko) {
+  // class 4 (no unit stride on an operand's free or inner contracted index) goes to the
+  // blocked-K persistent kernel when the outer contracted index is long enough to fill a
+  // 4 × 4 k-block; else to the per-tile gather kernel (variant 1)
+  if (layout_cls == 4 && Ko >= 4 && gemm_variant() >= 5) return kGemmClassKB;
+  return layout_cls;
+}
+
 bool gemm_fused_dot_ok() { return gemm_variant() != 1; }
 
 cudaError_t launch_gemm_group(const GemmBatch *b, long long total_tiles, int cls, cudaStream_t st) {
@@ -886,6 +996,14 @@ cudaError_t launch_gemm_group(const GemmBatch *b, long long total_tiles, int cls
       e = cudaFuncSetAttribute(persistent_fn<2, 2, 32, 16, true, true>(c), cudaFuncAttributeMaxDynamicSharedMemorySize,
                                PCfg<64, 32>::SMEM);
       if (e != cudaSuccess) return e;
+      if (c == 0) {
+        e = cudaFuncSetAttribute(zgemm_persistent_kb<2, 2, 32, 16, true, true>,
+                                 cudaFuncAttributeMaxDynamicSharedMemorySize, PCfg<64, 32>::SMEM);
+        if (e != cudaSuccess) return e;
+        e = cudaFuncSetAttribute(zgemm_persistent_kb<2, 2, 32, 16, true, false>,
+                                 cudaFuncAttributeMaxDynamicSharedMemorySize, PCfg<64, 32>::SMEM);
+        if (e != cudaSuccess) return e;
+      }
     }
     attr_set = true;
   }
@@ -905,6 +1023,15 @@ cudaError_t launch_gemm_group(const GemmBatch *b, long long total_tiles, int cls
     const char *e = getenv("MICCO_GEMM_PHASE_NS");
     phase_ns = e ? atoi(e) : kGemmPhaseNs;
     if (phase_ns < 0) phase_ns = 0;
+  }
+  if (cls == kGemmClassKB) {  // blocked-K gather (variant 5 or 6; gemm_kernel_class)
+    if (variant == 6)
+      zgemm_persistent_kb<2, 2, 32, 16, true, false><<<(unsigned)grid, 128, PCfg<64, 32>::SMEM, st>>>(
+          *b, total_tiles, (unsigned)phase_ns);
+    else
+      zgemm_persistent_kb<2, 2, 32, 16, true, true><<<(unsigned)grid, 128, PCfg<64, 32>::SMEM, st>>>(
+          *b, total_tiles, (unsigned)phase_ns);
+    return cudaGetLastError();
   }
   if (variant == 2)
     persistent_fn<2, 2, 32, 32, false, false>(cls)<<<(unsigned)grid, 128, PCfg<64, 64>::SMEM, st>>>(*b, total_tiles,

@@ -72,13 +72,15 @@ static_assert(sizeof(GemmBatch) <= 32764 && sizeof(DotBatch) <= 32764, "kernel p
 
 // GEMM descriptors carry their operand-layout class (layout.h gemm_class): 0..3 = unit-stride
 // inner index for both operands (warp-specialized kernel), 4 = generic gather kernel.
-constexpr int kGemmClasses = 5;
+// 5 = class 4 on the blocked-K persistent kernel (gemm_kernel_class).
+constexpr int kGemmClassKB = 5, kGemmClasses = 6;
 
 // The GEMM kernel variant in use (env MICCO_GEMM, see kernels.cu) and its CTA tile (complex
 // elements) for a layout class; tilesM/tilesN of a descriptor must use this shape.
 int gemm_variant();
 void gemm_tile_shape(int cls, int *bm, int *bn);
 bool gemm_uses_3m(int cls);  // 3 DMMA products per complex MAC for this layout class
+int gemm_kernel_class(int layout_cls, int Ko);  // the launch class of a descriptor
 bool gemm_fused_dot_ok();    // the selected persistent GEMM has the fused-dot epilogue (4 warps/CTA)
 
 // Grouped launches: descs in device memory (all of one layout class); grid covers the tiles.

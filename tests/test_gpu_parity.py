@@ -93,6 +93,22 @@ def test_two_baryon_all_matchings(order):
     assert np.array_equal(vals, valso)
 
 
+@pytest.mark.parametrize("N", [4, 16])
+def test_two_baryon_blocked_k(N):
+    """Greedy two-baryon graphs at N = 4 and 16: every c = 2 contraction whose operands have
+    no unit stride on their free or inner contracted index runs on the blocked-K GEMM
+    (4 ko × 4 ki stages, kernels.cu zgemm_persistent_kb); N = 9 above leaves ragged blocks.
+    Bit-exact on integer inputs."""
+    wl = workloads.c4_two_baryon(n_combos=1, N=N, Lt=2, pool=2, order="greedy",
+                                 matchings=list(range(0, 720, 5)))
+    check(wl)
+    wli = workloads.c4_two_baryon(n_combos=1, N=N, Lt=2, pool=2, order="greedy", mode=MODE_INT3,
+                                  matchings=list(range(0, 720, 5)))
+    C, vals, _ = run_gpu(wli)
+    Co, valso = oracle.correlator(wli, return_values=True)
+    assert np.array_equal(vals, valso)
+
+
 def test_two_baryon_n64_sample():
     """C4 at its full tensor size (N = 64 baryons), a sample of matchings, Lt = 4."""
     wl = workloads.c4_two_baryon(n_combos=1, N=64, Lt=4, pool=2, order="chain",

@@ -245,3 +245,21 @@ def test_reorder_dry_run_leaves_dag_untouched_on_failure():
     ctx.add_graph([ids[1], ids[2], ids[0]], workloads.meson_cycle_edges(3), None)  # rotation: all hits
     st2, _ = ctx.plan(1, [0, 0, 0])
     assert st2["unique_tasks"] == st0["unique_tasks"] and st2["dedup_hits"] == st0["dedup_hits"] + 2
+
+
+def test_policy_study_modelled_time(tmp_path):
+    """tools/policy_study.py (SURVEY.md §8(d) scheduler comparison) on a small repetition-heavy
+    set: MICCO's modelled plan time and peer traffic do not exceed round-robin's."""
+    import json
+    import sys
+    sys.path.insert(0, str(Path(__file__).resolve().parent.parent / "tools"))
+    import policy_study
+    out = tmp_path / "ps.json"
+    policy_study.main(["--graphs", "300", "--N", "32", "--Lt", "8", "--rates", "0.9", "--gpus", "4",
+                       "--out", str(out)])
+    rows = json.loads(out.read_text())["rows"]
+    for dist in ("uniform", "gaussian"):
+        r = {x["policy"]: x for x in rows if x["dist"] == dist}
+        assert r["micco"]["model_s"] <= r["round_robin"]["model_s"]
+        assert r["micco"]["bytes_p2p"] <= r["round_robin"]["bytes_p2p"]
+        assert r["micco"]["cache_hits"] >= r["round_robin"]["cache_hits"]
