@@ -319,7 +319,7 @@ def main():
                    "setup_s": round(t_setup, 1)},
         "tflops": flops_step / (ms_per_step / 1e3) / 1e12,
         "cache_per_step": {k: s0[k] for k in ("evictions", "cache_hits", "bytes_h2d", "bytes_d2h", "bytes_p2p")},
-        "roofline": {"bound": "tensor", "kernel": "zgemm_dmma_kernel (grouped)", "achieved": achieved,
+        "roofline": {"bound": "tensor", "kernel": "zgemm_persistent (3M, grouped per layout class)", "achieved": achieved,
                      "peak": FP64_DMMA_PEAK_TFLOPS, "unit": "TFLOP/s", "frac": achieved / FP64_DMMA_PEAK_TFLOPS,
                      "peak_source": "measured FP64 DMMA microbenchmark (profiles/fp64_peak_r01.txt); "
                                     "MEASURED_PEAKS.json has no FP64 entry",

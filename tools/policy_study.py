@@ -16,7 +16,7 @@ hits, evictions, max/mean load and the host planning time (host_s).  The modelle
 not a measurement (the GPU box has one B200); bytes, hits and load balance are exact
 properties of the plans the executor replays.
 
-Run: python tools/policy_study.py [--graphs 2000] [--out profiles/policy_study_r01.json]
+Run: python tools/policy_study.py [--graphs 10000] [--out profiles/policy_study_r01.json]
 """
 import argparse
 import json
@@ -49,7 +49,7 @@ def plan(wl, policy, n_gpus, window, budget):
 
 def main(argv=None):
     ap = argparse.ArgumentParser()
-    ap.add_argument("--graphs", type=int, default=2000)
+    ap.add_argument("--graphs", type=int, default=10000)
     ap.add_argument("--N", type=int, default=128)
     ap.add_argument("--Lt", type=int, default=64)
     ap.add_argument("--window", type=int, default=64)
