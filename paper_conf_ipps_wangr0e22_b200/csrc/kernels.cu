@@ -757,10 +757,54 @@ __device__ __forceinline__ void cmac(double &sr, double &si, double2 a, double2 
   si += a.x * b.y + a.y * b.x;
 }
 
-constexpr int DOT_SMEM = 2 * 32 * 33 * 16;  // two 32×33 complex tiles (33.8 KB)
+constexpr int DOT_UNROLL = 2;  // mode-1 micro-block pairs in flight per thread
+
+// mode 1: s = Σ_o Σ_{y<Y} Σ_{x<X} A[o][y·sAy + x] · B[o][x·sBx + y]   (layout.cpp: sAx = sBy = 1)
+// Register-only transpose: a thread owns a 2×2 (y, x) micro-block and loads A[y..y+1][x..x+1]
+// and B[x..x+1][y..y+1], so every pair A[y][x]·B[x][y] meets in one thread.  A warp covers
+// 16 y × 8 x: each load instruction touches 8 whole 128-byte lines (the two 16-byte halves of
+// a thread's 32-byte sector come from the same line), so no byte fetched is wasted, and there
+// is no shared-memory staging and no barrier; DOT_UNROLL micro-blocks keep 8·DOT_UNROLL loads
+// in flight per thread.  Slices are < 2^31 elements (executor.cu guard): 32-bit offsets.
+__device__ __forceinline__ void zdot_mode1(const DotDesc &d, const double2 *__restrict__ A,
+                                           const double2 *__restrict__ B, int tid, double &sr, double &si) {
+  const int lane = tid & 31, w = tid >> 5;
+  const int ty = lane >> 2, tx = lane & 3;
+  const int X = d.X, Y = d.Y;
+  const int nxb = (X + 7) >> 3, per_o = ((Y + 15) >> 4) * nxb;
+  const int O1 = d.O[1], O2 = d.O[2];
+  const int nb = d.O[0] * O1 * O2 * per_o;
+  const int sAy = (int)d.sAy, sBx = (int)d.sBx;
+  constexpr int NW = DT / 32;
+  for (int b0 = w; b0 < nb; b0 += NW * DOT_UNROLL) {
+    double2 va[DOT_UNROLL][4], vb[DOT_UNROLL][4];
+#pragma unroll
+    for (int u = 0; u < DOT_UNROLL; ++u) {
+      const int b = b0 + u * NW;
+      const int o = b / per_o, r = b - o * per_o;
+      const int yb = r / nxb, xb = r - yb * nxb;
+      const int o2 = o % O2, o01 = o / O2, o1 = o01 % O1, o0 = o01 / O1;
+      const int offA = (int)(o0 * d.sAo[0] + o1 * d.sAo[1] + o2 * d.sAo[2]);
+      const int offB = (int)(o0 * d.sBo[0] + o1 * d.sBo[1] + o2 * d.sBo[2]);
+      const int y = yb * 16 + 2 * ty, x = xb * 8 + 2 * tx;
+      const bool in = b < nb;
+#pragma unroll
+      for (int i = 0; i < 2; ++i)
+#pragma unroll
+        for (int j = 0; j < 2; ++j) {
+          const bool v = in && y + i < Y && x + j < X;
+          va[u][2 * i + j] = v ? __ldg(A + offA + (y + i) * sAy + x + j) : make_double2(0.0, 0.0);
+          vb[u][2 * i + j] = v ? __ldg(B + offB + (x + j) * sBx + y + i) : make_double2(0.0, 0.0);
+        }
+    }
+#pragma unroll
+    for (int u = 0; u < DOT_UNROLL; ++u)
+#pragma unroll
+      for (int k = 0; k < 4; ++k) cmac(sr, si, va[u][k], vb[u][k]);
+  }
+}
 
 __device__ __forceinline__ void zdot_body(const DotDesc *__restrict__ descs, int n_desc) {
-  extern __shared__ __align__(16) double2 dsm[];
   __shared__ double red[2][DT / 32];
   // Slice-major CTA order (every task of the launch has Lt CTAs): the CTAs resident at any
   // moment cover a few slices of every dot, so an operand shared by several dots of the launch
@@ -773,39 +817,30 @@ __device__ __forceinline__ void zdot_body(const DotDesc *__restrict__ descs, int
   const double2 *A = d.A + t * d.sAt;
   const double2 *B = d.B ? d.B + t * d.sBt : nullptr;
   double sr = 0.0, si = 0.0;
-  const long long O0 = d.O[0], O1 = d.O[1], O2 = d.O[2];
-  const long long Ototal = O0 * O1 * O2;
-  if (d.mode == 0) {  // flat (outer, x) index, one element pair per thread per step
-    const long long X = d.X, total = Ototal * X;
+  if (d.mode == 0) {  // x runs contiguous in both operands: rows o, threads along x
+    const int X = d.X, O1 = d.O[1], O2 = d.O[2], Ot = d.O[0] * O1 * O2;
+    const int sAx = (int)d.sAx, sBx = (int)d.sBx;
+    if (X >= DT / 2) {
+      for (int o = 0; o < Ot; ++o) {
+        const int o2 = o % O2, o01 = o / O2, o1 = o01 % O1, o0 = o01 / O1;
+        const double2 *Ao = A + (o0 * d.sAo[0] + o1 * d.sAo[1] + o2 * d.sAo[2]);
+        const double2 *Bo = B + (o0 * d.sBo[0] + o1 * d.sBo[1] + o2 * d.sBo[2]);
+#pragma unroll 8
+        for (int x = tid; x < X; x += DT) cmac(sr, si, __ldg(Ao + x * sAx), __ldg(Bo + x * sBx));
+      }
+    } else {  // short runs: flat (o, x) index, 32-bit decode per element
+      const int total = Ot * X;
 #pragma unroll 4
-    for (long long e = tid; e < total; e += DT) {
-      const long long o = e / X, x = e - o * X;
-      const long long o2 = o % O2, o01 = o / O2, o1 = o01 % O1, o0 = o01 / O1;
-      const long long offA = o0 * d.sAo[0] + o1 * d.sAo[1] + o2 * d.sAo[2] + x * d.sAx;
-      const long long offB = o0 * d.sBo[0] + o1 * d.sBo[1] + o2 * d.sBo[2] + x * d.sBx;
-      cmac(sr, si, A[offA], B[offB]);
+      for (int e = tid; e < total; e += DT) {
+        const int o = e / X, x = e - o * X;
+        const int o2 = o % O2, o01 = o / O2, o1 = o01 % O1, o0 = o01 / O1;
+        const int offA = (int)(o0 * d.sAo[0] + o1 * d.sAo[1] + o2 * d.sAo[2]) + x * sAx;
+        const int offB = (int)(o0 * d.sBo[0] + o1 * d.sBo[1] + o2 * d.sBo[2]) + x * sBx;
+        cmac(sr, si, __ldg(A + offA), __ldg(B + offB));
+      }
     }
-  } else {  // mode 1: A contiguous along x, B along y (32×32 shared-memory transpose tiles)
-    double2 (*As)[33] = reinterpret_cast<double2 (*)[33]>(dsm);
-    double2 (*Bs)[33] = reinterpret_cast<double2 (*)[33]>(dsm + 32 * 33);
-    const int ty = tid >> 5, tx = tid & 31;
-    for (long long o = 0; o < Ototal; ++o) {
-      const long long o2 = o % O2, o01 = o / O2, o1 = o01 % O1, o0 = o01 / O1;
-      const double2 *Ao = A + o0 * d.sAo[0] + o1 * d.sAo[1] + o2 * d.sAo[2];
-      const double2 *Bo = B + o0 * d.sBo[0] + o1 * d.sBo[1] + o2 * d.sBo[2];
-      for (int y0 = 0; y0 < d.Y; y0 += 32)
-        for (int x0 = 0; x0 < d.X; x0 += 32) {
-          for (int r = ty; r < 32; r += DT / 32) {
-            const int y = y0 + r, x = x0 + tx;
-            As[r][tx] = (y < d.Y && x < d.X) ? Ao[(long long)y * d.sAy + (long long)x * d.sAx] : make_double2(0, 0);
-            const int xb = x0 + r, yb = y0 + tx;
-            Bs[r][tx] = (xb < d.X && yb < d.Y) ? Bo[(long long)xb * d.sBx + (long long)yb * d.sBy] : make_double2(0, 0);
-          }
-          __syncthreads();
-          for (int r = ty; r < 32; r += DT / 32) cmac(sr, si, As[r][tx], Bs[tx][r]);
-          __syncthreads();
-        }
-    }
+  } else {
+    zdot_mode1(d, A, B, tid, sr, si);
   }
   // deterministic block reduction: xor butterfly, then warps in order
 #pragma unroll
@@ -1051,13 +1086,7 @@ cudaError_t launch_dot_group(const DotBatch *b, long long total_ctas, int cls, c
     zdot_warp_kernel<<<(unsigned)((total_ctas + DW - 1) / DW), DT, 0, st>>>(*b, total_ctas);
     return cudaGetLastError();
   }
-  static bool attr = false;
-  if (!attr) {
-    cudaError_t e = cudaFuncSetAttribute(zdot_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, DOT_SMEM);
-    if (e != cudaSuccess) return e;
-    attr = true;
-  }
-  zdot_kernel<<<(unsigned)total_ctas, DT, DOT_SMEM, st>>>(*b);
+  zdot_kernel<<<(unsigned)total_ctas, DT, 0, st>>>(*b);
   return cudaGetLastError();
 }
 

@@ -182,6 +182,49 @@ def test_c3_sampled_n256():
     check(wl.subset(list(range(12))))
 
 
+def sampled_check(wl, n_sample, seed=0, **kw):
+    """Run the whole workload through the library, then check a seeded sample of graph
+    values (the oracle computes each sampled graph on its own) and the full correlator's
+    consistency with the library's own per-graph values."""
+    ctx = M.Context(**kw)
+    M.load_workload(ctx, wl)
+    ctx.execute(1)
+    C = ctx.correlator()
+    rng = np.random.default_rng(seed)
+    sample = sorted(int(x) for x in rng.choice(len(wl.graphs), n_sample, replace=False))
+    sub = wl.subset(sample)
+    _, valso = oracle.correlator(sub, return_values=True)
+    for i, g in enumerate(sample):
+        v = np.array([ctx.graph_value(g, t) for t in range(wl.Lt)])
+        assert rel_err(v, valso[i]) <= TOL, g
+    vals = np.array([[ctx.graph_value(g, t) for t in range(wl.Lt)] for g in range(len(wl.graphs))])
+    coefs = np.array([complex(g.coef) for g in wl.graphs])
+    Csum = (coefs[:, None] * vals).sum(axis=0)
+    scale = (np.abs(coefs[:, None]) * np.abs(vals)).sum(axis=0)
+    assert np.max(np.abs(C - Csum) / scale) <= 1e-13
+    st = ctx.stats()
+    ctx.close()
+    return st
+
+
+def test_c3_full_size_sampled():
+    """C3 at its full tensor sizes (N = 256, Lt = 128) in the bench's launch configuration
+    (reuse-aware order, windows, grouped 3M launches with the fused final dot): 300 graphs,
+    5 sampled graph values against the oracle computed graph by graph."""
+    wl = workloads.c3_multi_meson(n_graphs=300, N=256, Lt=128, pool=6)
+    st = sampled_check(wl, 5, reorder=True)
+    assert st["n_gemm"] > 0
+
+
+def test_c4_full_size_sampled():
+    """C4 at its full sizes (N = 64 rank-3 baryons, Lt = 64) in the bench's launch
+    configuration (greedy order: c = 2 GETTs with K = 4096 on the persistent and blocked-K
+    kernels, then 64×64 dots): one sink/source combination's 720 matchings, 4 sampled."""
+    wl = workloads.c4_two_baryon(n_combos=1, N=64, Lt=64, pool=2, order="greedy")
+    st = sampled_check(wl, 4, seed=1)
+    assert st["n_gemm"] > 0
+
+
 def test_multiprocess_mode_single_rank_nccl():
     """The one-process-per-GPU path (plan replay of this rank's ops, NCCL communicator,
     ncclAllReduce of the scalar table) with world size 1: same C(t) bit for bit."""
