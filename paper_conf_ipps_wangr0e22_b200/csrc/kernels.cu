@@ -757,15 +757,26 @@ __device__ __forceinline__ void cmac(double &sr, double &si, double2 a, double2 
   si += a.x * b.y + a.y * b.x;
 }
 
+#ifndef MICCO_DOT_MINB
+#define MICCO_DOT_MINB 3  // resident dot CTAs per SM the register budget is sized for
+#endif
 constexpr int DOT_UNROLL = 2;  // mode-1 micro-block pairs in flight per thread
+
+// 32 bytes (two complex elements) in one LDG.E.256 (sm_100); p must be 32-byte aligned
+__device__ __forceinline__ void ldg_pair(const double2 *p, double2 &a, double2 &b) {
+  asm("ld.global.nc.v4.f64 {%0, %1, %2, %3}, [%4];" : "=d"(a.x), "=d"(a.y), "=d"(b.x), "=d"(b.y) : "l"(p));
+}
 
 // mode 1: s = Σ_o Σ_{y<Y} Σ_{x<X} A[o][y·sAy + x] · B[o][x·sBx + y]   (layout.cpp: sAx = sBy = 1)
 // Register-only transpose: a thread owns a 2×2 (y, x) micro-block and loads A[y..y+1][x..x+1]
-// and B[x..x+1][y..y+1], so every pair A[y][x]·B[x][y] meets in one thread.  A warp covers
-// 16 y × 8 x: each load instruction touches 8 whole 128-byte lines (the two 16-byte halves of
-// a thread's 32-byte sector come from the same line), so no byte fetched is wasted, and there
-// is no shared-memory staging and no barrier; DOT_UNROLL micro-blocks keep 8·DOT_UNROLL loads
-// in flight per thread.  Slices are < 2^31 elements (executor.cu guard): 32-bit offsets.
+// and B[x..x+1][y..y+1], so every pair A[y][x]·B[x][y] meets in one thread: no shared-memory
+// staging, no barrier.  A warp covers 16 y × 8 x, so each load instruction reads 8 whole
+// 128-byte lines.  V256 (every row start and x even, pointers 32-byte aligned): a thread's
+// two elements of a row come in one 32-byte LDG.E.256 — half the load instructions and L1
+// wavefronts of two 16-byte loads, whose half-sector pattern kept l1tex 92% busy on C4.
+// DOT_UNROLL blocks keep 4·DOT_UNROLL (V256) or 8·DOT_UNROLL loads in flight per thread.
+// Slices are < 2^31 elements (executor.cu guard): 32-bit offsets.
+template <bool V256>
 __device__ __forceinline__ void zdot_mode1(const DotDesc &d, const double2 *__restrict__ A,
                                            const double2 *__restrict__ B, int tid, double &sr, double &si) {
   const int lane = tid & 31, w = tid >> 5;
@@ -788,14 +799,27 @@ __device__ __forceinline__ void zdot_mode1(const DotDesc &d, const double2 *__re
       const int offB = (int)(o0 * d.sBo[0] + o1 * d.sBo[1] + o2 * d.sBo[2]);
       const int y = yb * 16 + 2 * ty, x = xb * 8 + 2 * tx;
       const bool in = b < nb;
-#pragma unroll
-      for (int i = 0; i < 2; ++i)
-#pragma unroll
-        for (int j = 0; j < 2; ++j) {
-          const bool v = in && y + i < Y && x + j < X;
-          va[u][2 * i + j] = v ? __ldg(A + offA + (y + i) * sAy + x + j) : make_double2(0.0, 0.0);
-          vb[u][2 * i + j] = v ? __ldg(B + offB + (x + j) * sBx + y + i) : make_double2(0.0, 0.0);
+      if constexpr (V256) {  // X, Y even: the pair (x, x + 1) is in or out together
+        const bool v = in && y < Y && x < X;
+        const double2 z = make_double2(0.0, 0.0);
+        va[u][0] = va[u][1] = va[u][2] = va[u][3] = z;
+        vb[u][0] = vb[u][1] = vb[u][2] = vb[u][3] = z;
+        if (v) {
+          ldg_pair(A + offA + y * sAy + x, va[u][0], va[u][1]);        // A[y][x], A[y][x+1]
+          ldg_pair(A + offA + (y + 1) * sAy + x, va[u][2], va[u][3]);  // A[y+1][x], A[y+1][x+1]
+          ldg_pair(B + offB + x * sBx + y, vb[u][0], vb[u][2]);        // B[x][y], B[x][y+1]
+          ldg_pair(B + offB + (x + 1) * sBx + y, vb[u][1], vb[u][3]);  // B[x+1][y], B[x+1][y+1]
         }
+      } else {
+#pragma unroll
+        for (int i = 0; i < 2; ++i)
+#pragma unroll
+          for (int j = 0; j < 2; ++j) {
+            const bool v = in && y + i < Y && x + j < X;
+            va[u][2 * i + j] = v ? __ldg(A + offA + (y + i) * sAy + x + j) : make_double2(0.0, 0.0);
+            vb[u][2 * i + j] = v ? __ldg(B + offB + (x + j) * sBx + y + i) : make_double2(0.0, 0.0);
+          }
+      }
     }
 #pragma unroll
     for (int u = 0; u < DOT_UNROLL; ++u)
@@ -840,7 +864,12 @@ __device__ __forceinline__ void zdot_body(const DotDesc *__restrict__ descs, int
       }
     }
   } else {
-    zdot_mode1(d, A, B, tid, sr, si);
+    // 32-byte pair loads need even row starts and x; the descriptor fixes this per dot
+    const bool v256 = ((((unsigned long long)A | (unsigned long long)B) & 31ull) == 0) &&
+                      (((d.X | d.Y | d.sAy | d.sBx | d.sAo[0] | d.sAo[1] | d.sAo[2] | d.sBo[0] | d.sBo[1] |
+                         d.sBo[2]) & 1) == 0);
+    if (v256) zdot_mode1<true>(d, A, B, tid, sr, si);
+    else zdot_mode1<false>(d, A, B, tid, sr, si);
   }
   // deterministic block reduction: xor butterfly, then warps in order
 #pragma unroll
@@ -974,7 +1003,7 @@ void (*persistent_fn(int cls))(const GemmBatch, long long, unsigned) {
   }
 }
 
-__global__ void __launch_bounds__(DT) zdot_kernel(const __grid_constant__ DotBatch b) { zdot_body(b.d, b.n); }
+__global__ void __launch_bounds__(DT, MICCO_DOT_MINB) zdot_kernel(const __grid_constant__ DotBatch b) { zdot_body(b.d, b.n); }
 __global__ void __launch_bounds__(DT) zdot_warp_kernel(const __grid_constant__ DotBatch b, long long items) {
   zdot_warp_body(b.d, b.n, items);
 }
