@@ -6,9 +6,11 @@
 // tensors of their connected components and their coefficient.
 #pragma once
 
+#include <condition_variable>
 #include <cstdint>
 #include <cstring>
 #include <memory>
+#include <mutex>
 #include <string>
 #include <map>
 #include <unordered_map>
@@ -213,7 +215,40 @@ enum { BOUNDS_FIXED = 0, BOUNDS_STAGE_SWEEP = 1, BOUNDS_REGRESSION = 2 };
 void predict_bounds(const double *features, int32_t out[3]);  // bounds_model.cpp
 void predict_bounds_raw(const double *features, double out[3]);
 
+// Op stream from a planner thread to the executor (executor.cu): make_plan publishes the
+// fused-dot table before its first stage and every stage's ops once they are final, so the
+// executor enqueues stage s while stage s+1 is being planned and the GPU does not wait for
+// the whole plan (every rank plans the whole DAG, so planning grows with the GPU count).
+struct PlanStream {
+  std::mutex m;
+  std::condition_variable cv;
+  std::vector<PlanOp> q;           // published, not yet taken by the executor
+  std::vector<int32_t> fused_dot;  // valid once have_fused
+  bool have_fused = false, done = false;
+  size_t published = 0;            // plan.ops already copied into q (planner side)
+  void publish_fused(const std::vector<int32_t> &f) {
+    std::lock_guard<std::mutex> lk(m);
+    fused_dot = f;
+    have_fused = true;
+    cv.notify_all();
+  }
+  void publish_ops(const std::vector<PlanOp> &ops) {
+    if (ops.size() == published) return;
+    std::lock_guard<std::mutex> lk(m);
+    q.insert(q.end(), ops.begin() + (long)published, ops.end());
+    published = ops.size();
+    cv.notify_all();
+  }
+  void finish() {
+    std::lock_guard<std::mutex> lk(m);
+    done = true;
+    have_fused = true;
+    cv.notify_all();
+  }
+};
+
 struct PlanInput {
+  PlanStream *stream = nullptr;                     // optional: publish ops as stages complete
   int32_t n_gpus;
   int32_t policy;
   int32_t reuse_bound[3];

@@ -23,6 +23,8 @@
 #include <cstdlib>
 #include <cstring>
 #include <string>
+#include <exception>
+#include <thread>
 #include <type_traits>
 #include <unordered_map>
 
@@ -174,6 +176,7 @@ struct Executor::Impl {
   std::unique_ptr<DotBatch> dot_batch{new DotBatch};
   int32_t chosen_bd[3] = {0, 0, 0};
   int chosen_bd_n = 0;
+  int stream_ok_n = 0;  // GPU count of the last completed execute (its nodes are materialised)
   // results on device 0
   double2 *d_vals = nullptr;
   size_t vals_elems = 0;
@@ -330,6 +333,7 @@ struct Executor::Impl {
   const double *host_src(int32_t x) const {
     const TensorRec &t = c.tensors[x];
     if (t.node >= 0) {
+      if (!c.nodes[t.node].host) materialize_nodes(c, {t.node});  // (streamed plans only)
       if (!c.nodes[t.node].host) fail(MICCO_ERR_STATE, "executor: node data not materialised");
       return c.nodes[t.node].host;
     }
@@ -644,32 +648,64 @@ struct Executor::Impl {
             in.initial_nodes[i].push_back(fn.first);
           }
     Plan plan;
+    bool sweep = false;  // whole-plan bound sweep (27 plans): synchronous
     if (!bd && c.opt.bound_model != BOUNDS_FIXED) {  // per-vector bounds (sweep or regression)
       in.bound_mode = c.opt.bound_model;
       for (int i = 0; i < 3; ++i) in.reuse_bound[i] = 0;
-      plan = make_plan(c, in);
     } else if (bd) {
       for (int i = 0; i < 3; ++i) in.reuse_bound[i] = bd[i];
-      plan = make_plan(c, in);
     } else if (chosen_bd_n == n) {  // bounds chosen by an earlier sweep for this GPU count
       for (int i = 0; i < 3; ++i) in.reuse_bound[i] = chosen_bd[i];
-      plan = make_plan(c, in);
     } else {
-      plan = make_plan_auto(c, in);
-      for (int i = 0; i < 3; ++i) chosen_bd[i] = plan.reuse_bound[i];
-      chosen_bd_n = n;
+      sweep = true;
     }
-    cached_nodes = plan.final_nodes;
-    fused_dot = plan.fused_dot;
-    {  // synthetic nodes this process uploads must have host data (lazy in multi-process mode)
+    // Streamed planning: once an execute on this GPU count has materialised the synthetic
+    // nodes this process uploads, later executes plan on a host thread and replay each stage
+    // as soon as it is final (PlanStream), so the GPU starts after the first stage is planned
+    // instead of the whole DAG (every rank plans the whole DAG: the plan grows with n).
+    const char *nps = getenv("MICCO_NO_PLAN_STREAM");
+    const bool streaming = !sweep && stream_ok_n == n && !(nps && nps[0] == '1');
+    PlanStream ps;
+    std::thread planner;
+    std::exception_ptr plan_err;
+    double plan_ms = 0;
+    if (streaming) {
+      in.stream = &ps;
+      planner = std::thread([&] {
+        auto p0 = std::chrono::steady_clock::now();
+        try {
+          plan = make_plan(c, in);
+          ps.publish_ops(plan.ops);
+        } catch (...) {
+          plan_err = std::current_exception();
+        }
+        plan_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - p0).count();
+        ps.finish();
+      });
+    } else {
+      if (sweep) {
+        plan = make_plan_auto(c, in);
+        for (int i = 0; i < 3; ++i) chosen_bd[i] = plan.reuse_bound[i];
+        chosen_bd_n = n;
+      } else {
+        plan = make_plan(c, in);
+      }
+      cached_nodes = plan.final_nodes;
+      fused_dot = plan.fused_dot;
+      // synthetic nodes this process uploads must have host data (lazy in multi-process mode)
       std::vector<int32_t> need;
       for (const PlanOp &op : plan.ops)
         if (op.kind == PlanOp::H2D && g[op.gpu].local && c.tensors[op.id].node >= 0 &&
             !c.nodes[c.tensors[op.id].node].host)
           need.push_back(c.tensors[op.id].node);
       materialize_nodes(c, need);
+      plan_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
     }
-    auto t1 = std::chrono::steady_clock::now();
+    // the planner thread must be joined on every exit path
+    struct Joiner {
+      std::thread &t;
+      ~Joiner() { if (t.joinable()) t.join(); }
+    } joiner{planner};
 
     micco_stats st{};
     st.struct_size = sizeof(st);
@@ -697,7 +733,31 @@ struct Executor::Impl {
         }
     }
     auto tq0 = std::chrono::steady_clock::now();
-    for (const PlanOp &op : plan.ops) run_op(op, st);
+    if (streaming) {
+      {
+        std::unique_lock<std::mutex> lk(ps.m);
+        ps.cv.wait(lk, [&] { return ps.have_fused; });
+        fused_dot = ps.fused_dot;
+      }
+      std::vector<PlanOp> batch;
+      for (;;) {
+        bool fin;
+        {
+          std::unique_lock<std::mutex> lk(ps.m);
+          ps.cv.wait(lk, [&] { return !ps.q.empty() || ps.done; });
+          batch.swap(ps.q);
+          fin = ps.done;  // finish() follows the last publish: nothing can arrive after this
+        }
+        for (const PlanOp &op : batch) run_op(op, st);
+        batch.clear();
+        if (fin) break;
+      }
+      planner.join();
+      if (plan_err) std::rethrow_exception(plan_err);
+      cached_nodes = plan.final_nodes;
+    } else {
+      for (const PlanOp &op : plan.ops) run_op(op, st);
+    }
     st.enqueue_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - tq0).count();
     st.host_pinned = c.arena.pinned() ? 1 : 0;
     for (auto &l : g)
@@ -795,7 +855,8 @@ struct Executor::Impl {
       else if (tm.kind == 1) { st.dot_kernel_ms += ms; ++st.dot_launches; }
     }
     st.wall_ms = std::chrono::duration<double, std::milli>(t2 - t0).count();
-    st.sched_ms = std::chrono::duration<double, std::milli>(t1 - t0).count();
+    st.sched_ms = plan_ms;  // planning time (overlapped with the replay when streamed)
+    stream_ok_n = n;
     st.evictions = plan.evictions;
     st.cache_hits = plan.cache_hits;
     st.unique_tasks = (int64_t)c.tasks.size();

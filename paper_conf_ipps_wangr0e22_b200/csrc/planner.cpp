@@ -445,6 +445,7 @@ Plan make_plan(const Context &ctx, const PlanInput &in) {
 
   const bool per_stage = in.bound_mode != BOUNDS_FIXED && n > 1 && in.policy == MICCO_POLICY_MICCO;
   double predicted = 0;
+  if (in.stream) in.stream->publish_fused(plan.fused_dot);
   for (int32_t s = 0; s < (int32_t)stages.size(); ++s) {
     double f[kBoundFeatures];
     stage_features(s, f);
@@ -470,6 +471,7 @@ Plan make_plan(const Context &ctx, const PlanInput &in) {
     sched.set_bounds(bd);
     plan.stage_bounds.insert(plan.stage_bounds.end(), bd, bd + 3);
     predicted += run_stage(s);
+    if (in.stream) in.stream->publish_ops(plan.ops);  // this stage's ops are final
   }
   if (in.keep_inputs)
     for (int32_t x = 0; x < NT; ++x)

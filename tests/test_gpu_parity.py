@@ -271,3 +271,28 @@ def test_reorder_parity():
     for n in (2, 4):
         C, _, _ = run_gpu(wl, n, [1, 2, 0], reorder=True, window_graphs=16)
         assert np.array_equal(C, ref), n
+
+
+def test_streamed_planning_bitwise(monkeypatch):
+    """Streamed planning (executor.cu PlanStream: the planner thread publishes each stage's
+    ops while earlier stages are replayed) gives the same C(t), bit for bit, as replaying a
+    finished plan — on 1 and 3 logical GPUs, with cached and with released node replicas."""
+    wl = workloads.c3_multi_meson(n_graphs=80, N=40, Lt=3, pool=4)
+    Co = oracle.correlator(wl)
+    for n in (1, 3):
+        res = {}
+        for mode in ("0", "1"):
+            monkeypatch.setenv("MICCO_NO_PLAN_STREAM", mode)
+            ctx = M.Context(keep_inputs_resident=True, window_graphs=8)
+            M.load_workload(ctx, wl)
+            out = []
+            for rep in range(3):  # first execute plans synchronously; later ones stream
+                if rep == 2:
+                    ctx.release_cache()
+                ctx.execute(n, [1, 1, 0] if n > 1 else None)
+                out.append(ctx.correlator())
+            ctx.close()
+            res[mode] = out
+        for a, b in zip(res["0"], res["1"]):
+            assert np.array_equal(a, b), n
+        assert rel_err(res["0"][-1], Co) <= TOL
