@@ -324,6 +324,8 @@ Plan host_plan(Context &c, int32_t n_gpus, const int32_t *reuse_bound, int32_t b
   in.host_gbs = 55;
   in.flops_per_s = 30e12;
   if (bound_mode < 0) bound_mode = reuse_bound ? BOUNDS_FIXED : c.opt.bound_model;
+  if (bound_mode != BOUNDS_FIXED) in.bound_mode = bound_mode;
+  in.window_graphs = choose_window(c, in);
   if (bound_mode != BOUNDS_FIXED) {
     in.bound_mode = bound_mode;
     return make_plan(c, in);

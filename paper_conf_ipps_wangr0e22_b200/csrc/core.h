@@ -263,5 +263,8 @@ struct PlanInput {
 
 Plan make_plan(const Context &ctx, const PlanInput &in);
 Plan make_plan_auto(const Context &ctx, PlanInput in);  // sweeps reuse bounds when asked
+// window_graphs when options.window_graphs == 0: the largest window the budget allows
+// without extra host traffic (planner.cpp)
+int32_t choose_window(const Context &ctx, PlanInput in);
 
 }  // namespace micco

@@ -177,6 +177,9 @@ struct Executor::Impl {
   int32_t chosen_bd[3] = {0, 0, 0};
   int chosen_bd_n = 0;
   int stream_ok_n = 0;  // GPU count of the last completed execute (its nodes are materialised)
+  int32_t chosen_w = 256;  // window chosen by choose_window for chosen_w_n GPUs
+  int chosen_w_n = 0;
+  int64_t cache_dag_key = -1;
   // results on device 0
   double2 *d_vals = nullptr;
   size_t vals_elems = 0;
@@ -649,15 +652,28 @@ struct Executor::Impl {
           }
     Plan plan;
     bool sweep = false;  // whole-plan bound sweep (27 plans): synchronous
+    // choices cached across executes are valid for this GPU count and this DAG
+    const int64_t dag_key = (int64_t)c.tasks.size() * 1000003 + (int64_t)c.graphs.size();
+    if (dag_key != cache_dag_key) {
+      chosen_bd_n = chosen_w_n = 0;
+      cache_dag_key = dag_key;
+    }
+    for (int i = 0; i < 3; ++i) in.reuse_bound[i] = 0;
     if (!bd && c.opt.bound_model != BOUNDS_FIXED) {  // per-vector bounds (sweep or regression)
       in.bound_mode = c.opt.bound_model;
-      for (int i = 0; i < 3; ++i) in.reuse_bound[i] = 0;
     } else if (bd) {
       for (int i = 0; i < 3; ++i) in.reuse_bound[i] = bd[i];
     } else if (chosen_bd_n == n) {  // bounds chosen by an earlier sweep for this GPU count
       for (int i = 0; i < 3; ++i) in.reuse_bound[i] = chosen_bd[i];
     } else {
       sweep = true;
+    }
+    if (in.window_graphs <= 0) {  // options.window_graphs == 0: sized to the budget
+      if (chosen_w_n != n) {
+        chosen_w = choose_window(c, in);
+        chosen_w_n = n;
+      }
+      in.window_graphs = chosen_w;
     }
     // Streamed planning: once an execute on this GPU count has materialised the synthetic
     // nodes this process uploads, later executes plan on a host thread and replay each stage

@@ -484,6 +484,32 @@ Plan make_plan(const Context &ctx, const PlanInput &in) {
   return plan;
 }
 
+int32_t choose_window(const Context &ctx, PlanInput in) {
+  if (in.window_graphs > 0) return in.window_graphs;
+  // A window's stages are level-synchronous, so all the intermediates of its first level are
+  // live at once: under a tight budget a large window spills what a smaller one would not
+  // (C5 at 25 GB: W = 256 moves 178 GB over PCIe per execute, W = 128 0.4 GB).  Take the
+  // largest W in {256, 128, ..., 1} that a smaller W does not beat by more than 1% in the
+  // cost model (which prices host bytes); stop at the first plan that spills nothing and
+  // evicts nothing, since a smaller window cannot save bytes.  Stages stay as large as the
+  // budget allows (fewer, larger grouped launches).
+  in.stream = nullptr;
+  int32_t best_w = 256;
+  double best = 0;
+  bool have = false;
+  for (int32_t W = 256; W >= 1; W /= 2) {
+    in.window_graphs = W;
+    const Plan p = make_plan(ctx, in);
+    if (!have || p.predicted_s < best * 0.99) {
+      best = p.predicted_s;
+      best_w = W;
+      have = true;
+    }
+    if (p.bytes_d2h == 0 && p.evictions == 0) break;
+  }
+  return best_w;
+}
+
 Plan make_plan_auto(const Context &ctx, PlanInput in) {
   if (in.n_gpus == 1 || in.policy == MICCO_POLICY_ROUND_ROBIN || in.policy == MICCO_POLICY_LEAST_LOADED ||
       in.policy == MICCO_POLICY_MICCO_NAIVE) {
