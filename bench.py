@@ -46,7 +46,7 @@ def parse():
     ap.add_argument("--steps", type=int, default=5)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="micco", choices=["micco", "reference"])
-    ap.add_argument("--config", default="c2", choices=["c2", "c3", "c4", "c5"],
+    ap.add_argument("--config", default="c2", choices=["c2", "c3", "c4", "c5", "c5full"],
                     help="c2 = BASELINE configs[1] (the headline); c3 / c4 = configs[2] / [3] shapes")
     ap.add_argument("--graphs", type=int, default=10000, help="graphs per GPU (weak scaling)")
     ap.add_argument("--N", type=int, default=128)
@@ -117,6 +117,9 @@ def c2_workload(args, world):
     from micco_inputs import workloads
     if args.config == "c3":  # multi-meson: N = 256, Lt = 128 (BASELINE configs[2])
         return workloads.c3_multi_meson(n_graphs=args.graphs * world, N=256, Lt=128)
+    if args.config == "c5full":  # configs[4] at its stated size: N = 64 baryons, Lt = 64, rank-4
+        # intermediates of 17.2 GB, 1358 GB of intermediate demand against ~163 GB of HBM
+        return workloads.c5_mixed(n_combos=4, Nb=64, Nm=256, Lt=64, pool=4, meson_graphs=64)
     if args.config == "c5":  # oversubscribed mixed set (configs[4]), scaled to the host's RAM:
         # rank-4 N = 64 intermediates of 4.3 GB (Lt = 16) shared across the stream, plus C3-style
         # N = 256 meson graphs; unconstrained peak 37.6 GB, run against a 25 GB budget
