@@ -760,7 +760,10 @@ __device__ __forceinline__ void cmac(double &sr, double &si, double2 a, double2 
 #ifndef MICCO_DOT_MINB
 #define MICCO_DOT_MINB 3  // resident dot CTAs per SM the register budget is sized for
 #endif
-constexpr int DOT_UNROLL = 2;  // mode-1 micro-block pairs in flight per thread
+#ifndef MICCO_DOT_UNROLL
+#define MICCO_DOT_UNROLL 2
+#endif
+constexpr int DOT_UNROLL = MICCO_DOT_UNROLL;  // mode-1 micro-block pairs in flight per thread
 
 // 32 bytes (two complex elements) in one LDG.E.256 (sm_100); p must be 32-byte aligned
 __device__ __forceinline__ void ldg_pair(const double2 *p, double2 &a, double2 &b) {

@@ -76,10 +76,15 @@ struct PlanState {
     return it == u.end() ? std::numeric_limits<int32_t>::max() : *it;
   }
 
-  // Evict unpinned replicas on g until need more bytes fit; false if impossible.
+  // Evict unpinned replicas on g until need more bytes fit; false if impossible.  Dead and
+  // replicated tensors (classes 0, 1: no host traffic to evict) are evicted down to a low-water
+  // mark budget/64 below the need, so the scan-and-sort runs once per ~budget/64 bytes instead of
+  // once per allocation (a full 8-GPU C2 plan evicts ~17k replicas: 17 s → 0.2 s of planning);
+  // sole copies (class 2, a D2H spill) only to fit the need itself.
   bool make_room(int g, int64_t need) {
     const int64_t budget = in.budget[g];
     if (mem[g] + need <= budget) return true;
+    const int64_t low = budget - budget / 64;
     struct Cand { int cls; int32_t next; int32_t x; };
     std::vector<Cand> cands;
     for (int32_t x : res[g]) {
@@ -96,7 +101,7 @@ struct PlanState {
       return a.x < b.x;
     });
     for (const Cand &c : cands) {
-      if (mem[g] + need <= budget) break;
+      if (mem[g] + need <= (c.cls == 2 ? budget : low)) break;
       if (c.cls == 2) {  // sole copy: spill to pinned host memory first
         emit(PlanOp::SPILL, g, -1, c.x);
         on_host[c.x] = 1;
@@ -490,8 +495,8 @@ int32_t choose_window(const Context &ctx, PlanInput in) {
   // live at once: under a tight budget a large window spills what a smaller one would not
   // (C5 at 25 GB: W = 256 moves 178 GB over PCIe per execute, W = 128 0.4 GB).  Take the
   // largest W in {256, 128, ..., 1} that a smaller W does not beat by more than 1% in the
-  // cost model (which prices host bytes); stop at the first plan that spills nothing and
-  // evicts nothing, since a smaller window cannot save bytes.  Stages stay as large as the
+  // cost model (which prices host bytes); stop at the first plan that spills nothing (a smaller
+  // window only bounds the live set of intermediates).  Stages stay as large as the
   // budget allows (fewer, larger grouped launches).
   in.stream = nullptr;
   int32_t best_w = 256;
@@ -505,7 +510,7 @@ int32_t choose_window(const Context &ctx, PlanInput in) {
       best_w = W;
       have = true;
     }
-    if (p.bytes_d2h == 0 && p.evictions == 0) break;
+    if (p.bytes_d2h == 0) break;  // no spill (evicting dead or replicated tensors is cheap)
   }
   return best_w;
 }
