@@ -16,7 +16,8 @@ grouped complex-FP64 DMMA GEMMs and dots → per-graph finalize → C(t) on the 
   by CUDA events on its launching stream inside the library, against the measured FP64
   DMMA peak (profiles/fp64_peak_r01.txt).
 * cpu_baseline: the CPU oracle (oracle/) on a bounded sample of the same graphs.
-Multi-GPU (torchrun, one process per GPU): weak scaling, N × 10k graphs; the plan is built
+Multi-GPU (torchrun, one process per GPU): weak scaling, N independent 10k-graph C2 sets
+(disjoint node pools, interleaved graph by graph; set 0 is the N = 1 workload); the plan is built
 identically on every rank, operands move with ncclSend/ncclRecv, one ncclAllReduce
 combines the per-graph scalars.  Timing: barrier + cuda.synchronize on both sides, CUDA
 events, max over ranks.
@@ -126,7 +127,11 @@ def c2_workload(args, world):
         return workloads.c5_mixed(n_combos=1, Nb=64, Nm=256, Lt=16, pool=2, meson_graphs=64)
     if args.config == "c4":  # two-baryon: rank-3 N = 64, Lt = 64 (configs[3]); graphs = combos × 720
         return workloads.c4_two_baryon(n_combos=max(1, args.graphs * world // 720), N=64, Lt=64, order="greedy")
-    return workloads.c2_meson_set(n_graphs=args.graphs * world, N=args.N, Lt=args.Lt, rate=args.rate,
+    if world > 1:  # weak scaling: one independent 10k-graph C2 set per GPU, interleaved in one
+        # stream (set 0 is the N = 1 workload); the scheduler is not told the partition
+        return workloads.c2_weak_sets(world, n_graphs=args.graphs, N=args.N, Lt=args.Lt, rate=args.rate,
+                                      dist=args.dist, seed=2)
+    return workloads.c2_meson_set(n_graphs=args.graphs, N=args.N, Lt=args.Lt, rate=args.rate,
                                   dist=args.dist, seed=2)
 
 

@@ -134,6 +134,28 @@ def c2_meson_set(n_graphs: int = 10000, N: int = 128, Lt: int = 64, rate: float 
                     {"N": N, "rate": rate, "dist": dist})
 
 
+def c2_weak_sets(n_sets: int, n_graphs: int = 10000, N: int = 128, Lt: int = 64, rate: float = 0.9,
+                 dist: str = "uniform", seed: int = 2, mode: int = MODE_UNIFORM) -> Workload:
+    """Weak scaling of C2 over n_sets GPUs: n_sets independent C2 sets (seeds seed .. seed +
+    n_sets − 1, disjoint node pools) in one graph stream, interleaved graph by graph.  Set 0 is
+    exactly c2_meson_set(seed=seed).  The library is not told the partition: the scheduler
+    must find it through operand reuse (Alg. 1)."""
+    sets = [c2_meson_set(n_graphs, N, Lt, rate, dist, seed + s, mode) for s in range(n_sets)]
+    nodes: List[NodeSpec] = []
+    base = []
+    for s, w in enumerate(sets):
+        base.append(len(nodes))
+        nodes += [NodeSpec(nd.rank, nd.N, nd.key + 1_000_000 * s) for nd in w.nodes]
+    graphs = []
+    for i in range(n_graphs):
+        for s, w in enumerate(sets):
+            g = w.graphs[i]
+            graphs.append(GraphSpec([base[s] + x for x in g.inst], list(g.edges),
+                                    None if g.order is None else list(g.order), g.coef))
+    name = sets[0].name if n_sets == 1 else f"{sets[0].name}_x{n_sets}sets"
+    return Workload(name, Lt, seed, mode, nodes, graphs, {"N": N, "rate": rate, "dist": dist, "sets": n_sets})
+
+
 # ---------------------------------------------------------------- C3
 
 

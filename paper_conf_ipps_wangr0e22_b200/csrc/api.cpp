@@ -326,6 +326,17 @@ Plan host_plan(Context &c, int32_t n_gpus, const int32_t *reuse_bound, int32_t b
   if (bound_mode < 0) bound_mode = reuse_bound ? BOUNDS_FIXED : c.opt.bound_model;
   if (bound_mode != BOUNDS_FIXED) in.bound_mode = bound_mode;
   in.window_graphs = choose_window(c, in);
+  const char *warm = getenv("MICCO_PLAN_WARM");  // tools: plan a repeat execute (keep_inputs
+  if (warm && warm[0] == '1' && in.keep_inputs) {  // replicas left by a first, cold one)
+    Plan cold = reuse_bound || bound_mode != BOUNDS_FIXED ? make_plan(c, in) : make_plan_auto(c, in);
+    in.initial_nodes.assign(n_gpus, {});
+    for (const auto &fn : cold.final_nodes)
+      for (int g = 0; g < n_gpus; ++g)
+        if ((fn.second >> g) & 1) in.initial_nodes[g].push_back(fn.first);
+    if (!reuse_bound && bound_mode == BOUNDS_FIXED)
+      for (int i = 0; i < 3; ++i) in.reuse_bound[i] = cold.reuse_bound[i];
+    return make_plan(c, in);
+  }
   if (bound_mode != BOUNDS_FIXED) {
     in.bound_mode = bound_mode;
     return make_plan(c, in);

@@ -100,3 +100,45 @@ def test_c5_structure():
         partner = v if u == 0 else u
         shared = sum(1 for (a, _, b, _) in G.edges if {a, b} == {0, partner})
         assert shared == 1
+
+
+def test_c2_weak_sets_structure():
+    """bench.py's weak-scaling workload: set 0 is exactly the N = 1 C2 workload, the sets
+    have disjoint node pools, and graphs are interleaved set by set."""
+    from micco_inputs import workloads
+    one = workloads.c2_meson_set(n_graphs=50, N=8, Lt=2, rate=0.7, seed=2)
+    same = workloads.c2_weak_sets(1, n_graphs=50, N=8, Lt=2, rate=0.7, seed=2)
+    assert [n.key for n in same.nodes] == [n.key for n in one.nodes]
+    assert [g.inst for g in same.graphs] == [g.inst for g in one.graphs]
+    assert [g.coef for g in same.graphs] == [g.coef for g in one.graphs]
+    three = workloads.c2_weak_sets(3, n_graphs=50, N=8, Lt=2, rate=0.7, seed=2)
+    assert len(three.graphs) == 150
+    owner = {}
+    for i, g in enumerate(three.graphs):
+        for x in g.inst:
+            assert owner.setdefault(x, i % 3) == i % 3  # graph i belongs to set i % 3
+    keys = [n.key for n in three.nodes]
+    assert len(set(keys)) == len(keys)
+    s1 = workloads.c2_meson_set(n_graphs=50, N=8, Lt=2, rate=0.7, seed=3)
+    assert [len(g.inst) for g in three.graphs[1::3]] == [len(g.inst) for g in s1.graphs]
+
+
+def test_c2_weak_sets_plan_partitions():
+    """Host-only plans of the 4-GPU weak-scaling workload: the MICCO scheduler finds the
+    partition well enough that a repeat execute (replicas cached) moves no byte over PCIe
+    and evicts nothing, while load stays balanced."""
+    import os
+    import paper_conf_ipps_wangr0e22_b200 as M
+    from micco_inputs import workloads
+    wl = workloads.c2_weak_sets(4, n_graphs=300, N=8, Lt=2, rate=0.9, seed=2)
+    node_bytes = 8 * 8 * 2 * 16
+    ctx = M.Context(keep_inputs_resident=True, mem_budget_bytes=400 * node_bytes, dist_rank=0, dist_world=4)
+    M.load_workload(ctx, wl)
+    os.environ["MICCO_PLAN_WARM"] = "1"
+    try:
+        st, _ = ctx.plan(4, [2, 2, 2])
+    finally:
+        os.environ.pop("MICCO_PLAN_WARM")
+    ctx.close()
+    assert st["bytes_h2d"] == 0 and st["evictions"] == 0 and st["bytes_d2h"] == 0
+    assert st["max_over_mean_load"] < 1.1
