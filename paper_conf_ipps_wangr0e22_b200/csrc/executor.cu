@@ -142,6 +142,7 @@ struct LGpu {
   bool local = true;
   cudaStream_t st = nullptr;   // compute stream: kernels, P2P, spills, frees
   cudaStream_t cst = nullptr;  // copy stream: H2D prefetch (async, overlaps the kernels)
+  cudaStream_t pst = nullptr;  // peer stream: NVLink moves (peer copies / NCCL send-recv)
   std::vector<cudaEvent_t> flush_ev;  // compute-stream event after each flushed chunk
   std::vector<int64_t> chunk_fetch;   // bytes fetched for each flushed chunk
   std::vector<int64_t> fetch_bytes_since;
@@ -219,10 +220,13 @@ struct Executor::Impl {
       if (p) { cudaFreeAsync(p, l.st); p = nullptr; }
     cudaStreamSynchronize(l.st);
     if (l.cst) cudaStreamSynchronize(l.cst);
+    if (l.pst) cudaStreamSynchronize(l.pst);
     l.readers.clear();
     if (destroy_stream) {
       cudaStreamDestroy(l.st);
       cudaStreamDestroy(l.cst);
+      cudaStreamDestroy(l.pst);
+      l.pst = nullptr;
       l.st = nullptr;
       l.cst = nullptr;
     }
@@ -274,6 +278,7 @@ struct Executor::Impl {
       }
       CK(cudaStreamCreateWithFlags(&l.st, cudaStreamNonBlocking));
       CK(cudaStreamCreateWithFlags(&l.cst, cudaStreamNonBlocking));
+      CK(cudaStreamCreateWithFlags(&l.pst, cudaStreamNonBlocking));
     }
     if (dist()) {
       if (!c.have_nccl_id) fail(MICCO_ERR_STATE, "multi-process mode needs micco_set_nccl_id before execute");
@@ -306,8 +311,19 @@ struct Executor::Impl {
       int64_t usable = (int64_t)(fr * 0.92) - (2LL << 30);
       b[i] = std::max<int64_t>(usable / k, 1LL << 28);
     }
-    if (dist()) {  // every rank must plan with identical budgets
+    if (dist()) {  // every rank must plan with identical budgets: the minimum over ranks
       int64_t mn = *std::min_element(b.begin(), b.end());
+      if (c.opt.mem_budget_bytes <= 0 && comm) {
+        LGpu &l = g[my_rank()];
+        CK(cudaSetDevice(l.dev));
+        int64_t *d = nullptr;
+        CK(cudaMallocAsync((void **)&d, sizeof(int64_t), l.st));
+        CK(cudaMemcpyAsync(d, &mn, sizeof(int64_t), cudaMemcpyHostToDevice, l.st));
+        NK(nccl().AllReduce(d, d, 1, ncclInt64, ncclMin, comm, l.st));
+        CK(cudaMemcpyAsync(&mn, d, sizeof(int64_t), cudaMemcpyDeviceToHost, l.st));
+        CK(cudaFreeAsync(d, l.st));
+        CK(cudaStreamSynchronize(l.st));
+      }
       std::fill(b.begin(), b.end(), mn);
     }
     budget_cache = b;
@@ -317,12 +333,33 @@ struct Executor::Impl {
 
   // ---------------------------------------------------------------- op replay
 
-  cudaEvent_t record(int gi) {
+  cudaEvent_t record(int gi) { return record_on(gi, g[gi].st); }
+  cudaEvent_t record_on(int gi, cudaStream_t s) {
     LGpu &l = g[gi];
     cudaEvent_t e = devs[l.dev].sync_events.get();
     CK(cudaSetDevice(l.dev));
-    CK(cudaEventRecord(e, l.st));
+    CK(cudaEventRecord(e, s));
     return e;
+  }
+  // Peer moves run on their own stream (MICCO_P2P_STREAM=0: on the compute stream), ordered
+  // with the kernels by events only: the transfer overlaps the kernels of earlier stages, and
+  // in multi-process mode an ncclSend no longer holds the sender's compute stream until the
+  // receiver's stream reaches the matching ncclRecv.  All NCCL calls of a rank stay on one
+  // stream in the global plan order (the pairing argument of the op list is unchanged).
+  // A peer move for the chunk being built may start once the compute stream has finished the
+  // chunk before the last flushed one: the peer stream runs at most ~2 stages ahead, so
+  // replicas are not allocated far ahead of the frees the plan's budget assumed.
+  void pace_peer(LGpu &l) {
+    const size_t nf = l.flush_ev.size();
+    if (nf >= 2) CK(cudaStreamWaitEvent(l.pst, l.flush_ev[nf - 2], 0));
+  }
+  bool p2p_stream() const {
+    static int on = -1;
+    if (on < 0) {
+      const char *e = getenv("MICCO_P2P_STREAM");
+      on = (e && e[0] == '0') ? 0 : 1;
+    }
+    return on == 1;
   }
 
   double2 *alloc(LGpu &l, int64_t bytes) {
@@ -539,29 +576,46 @@ struct Executor::Impl {
         LGpu &dst = g[op.gpu];
         LGpu &src = g[op.src];
         const int64_t nb = bytes_of(op.id);
+        const bool ps = p2p_stream();
         if (dist()) {
           if (dst.local) {
             CK(cudaSetDevice(dst.dev));
-            double2 *p = alloc(dst, nb);
-            NK(nccl().Recv(p, (size_t)nb / 8, ncclDouble, op.src, comm, dst.st));
-            dst.ptr[op.id] = p;
+            cudaStream_t s = ps ? dst.pst : dst.st;
+            if (ps) pace_peer(dst);
+            void *p = nullptr;
+            CK(cudaMallocAsync(&p, (size_t)nb, s));
+            NK(nccl().Recv(p, (size_t)nb / 8, ncclDouble, op.src, comm, s));
+            if (ps) CK(cudaStreamWaitEvent(dst.st, record_on(op.gpu, s), 0));  // consumers wait
+            dst.ptr[op.id] = (double2 *)p;
             st.bytes_p2p += nb;
           } else if (src.local) {
             CK(cudaSetDevice(src.dev));
-            NK(nccl().Send(src.ptr[op.id], (size_t)nb / 8, ncclDouble, op.gpu, comm, src.st));
+            if (ps) {
+              CK(cudaStreamWaitEvent(src.pst, record(op.src), 0));  // the replica is complete
+              NK(nccl().Send(src.ptr[op.id], (size_t)nb / 8, ncclDouble, op.gpu, comm, src.pst));
+              src.readers[op.id].push_back(record_on(op.src, src.pst));  // a free waits for the send
+            } else {
+              NK(nccl().Send(src.ptr[op.id], (size_t)nb / 8, ncclDouble, op.gpu, comm, src.st));
+            }
           }
           return;
         }
         cudaEvent_t ready = record(op.src);  // the replica on src is complete
         CK(cudaSetDevice(dst.dev));
-        CK(cudaStreamWaitEvent(dst.st, ready, 0));
-        double2 *p = alloc(dst, nb);
+        cudaStream_t s = ps ? dst.pst : dst.st;
+        CK(cudaStreamWaitEvent(s, ready, 0));
+        if (ps) pace_peer(dst);
+        void *pv = nullptr;
+        CK(cudaMallocAsync(&pv, (size_t)nb, s));
+        double2 *p = (double2 *)pv;
         if (dst.dev == src.dev)
-          CK(cudaMemcpyAsync(p, src.ptr[op.id], nb, cudaMemcpyDeviceToDevice, dst.st));
+          CK(cudaMemcpyAsync(p, src.ptr[op.id], nb, cudaMemcpyDeviceToDevice, s));
         else
-          CK(cudaMemcpyPeerAsync(p, dst.dev, src.ptr[op.id], src.dev, nb, dst.st));
+          CK(cudaMemcpyPeerAsync(p, dst.dev, src.ptr[op.id], src.dev, nb, s));
+        cudaEvent_t done = record_on(op.gpu, s);
+        if (ps) CK(cudaStreamWaitEvent(dst.st, done, 0));
         dst.ptr[op.id] = p;
-        src.readers[op.id].push_back(record(op.gpu));
+        src.readers[op.id].push_back(done);
         st.bytes_p2p += nb;
         return;
       }
@@ -801,6 +855,8 @@ struct Executor::Impl {
       if (i != home && g[i].local) CK(cudaStreamWaitEvent(H.st, record(i), 0));
     double2 *S = devs[H.dev].scalars;
     if (dist()) {
+      // every NCCL call of this rank in one order: the all-reduce after the last send/recv
+      if (H.pst) CK(cudaStreamWaitEvent(H.st, record_on(home, H.pst), 0));
       NK(nccl().AllReduce(S, S, selems * 2, ncclDouble, ncclSum, comm, H.st));
     } else {
       for (int d = 0; d < ndev; ++d) {
@@ -851,6 +907,7 @@ struct Executor::Impl {
         CK(cudaSetDevice(l.dev));
         CK(cudaStreamSynchronize(l.st));
         CK(cudaStreamSynchronize(l.cst));
+        CK(cudaStreamSynchronize(l.pst));
       }
     auto t2 = std::chrono::steady_clock::now();
 
