@@ -263,3 +263,30 @@ def test_policy_study_modelled_time(tmp_path):
         assert r["micco"]["model_s"] <= r["round_robin"]["model_s"]
         assert r["micco"]["bytes_p2p"] <= r["round_robin"]["bytes_p2p"]
         assert r["micco"]["cache_hits"] >= r["round_robin"]["cache_hits"]
+
+
+def test_budget_sized_window():
+    """window_graphs = 0 (planner.cpp choose_window): under a budget a few rank-4
+    intermediates deep, the 256-graph window spills and re-fetches, while the chosen window
+    plans without any spill and with the fewest host bytes of the candidates tried; with
+    room to spare the default stays one 256-graph window."""
+    wl = workloads.c5_mixed(n_combos=1, Nb=8, Nm=12, Lt=2, pool=2, meson_graphs=12)
+    r4 = 8 ** 4 * 2 * 16
+    stats = {}
+    for W in (0, 256, 64, 16):
+        ctx = _ctx(mem_budget_bytes=4 * r4, window_graphs=W)
+        M.load_workload(ctx, wl)
+        stats[W], _ = ctx.plan(1, [0, 0, 0])
+        ctx.close()
+    assert stats[256]["bytes_d2h"] > 0 and stats[64]["bytes_d2h"] > 0
+    assert stats[0]["bytes_d2h"] == 0 and stats[0]["evictions"] == 0
+    assert stats[0]["bytes_h2d"] == min(s["bytes_h2d"] for s in stats.values())
+    roomy = _ctx(mem_budget_bytes=1 << 34, window_graphs=0)
+    M.load_workload(roomy, wl)
+    s0, _ = roomy.plan(1, [0, 0, 0])
+    roomy.close()
+    fixed = _ctx(mem_budget_bytes=1 << 34, window_graphs=256)
+    M.load_workload(fixed, wl)
+    s256, _ = fixed.plan(1, [0, 0, 0])
+    fixed.close()
+    assert s0["n_stages"] == s256["n_stages"] and s0["bytes_h2d"] == s256["bytes_h2d"]
