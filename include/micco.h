@@ -84,9 +84,14 @@ typedef struct {
   size_t struct_size;          /* sizeof(micco_options): ABI versioning */
   int64_t mem_budget_bytes;    /* per GPU (GPUMaxMemory); 0 = device free memory
                                   minus a 2 GiB reserve, split evenly between logical GPUs
-                                  sharing a device */
+                                  sharing a device (multi-process mode: the minimum over ranks,
+                                  agreed by an NCCL all-reduce, so every rank plans alike) */
   int32_t policy;              /* MICCO_POLICY_* */
-  int32_t window_graphs;       /* graphs per window (one stream of vectors); 0 = auto */
+  int32_t window_graphs;       /* graphs per window (one stream of vectors); 0 = auto: the largest
+                                  of 256, 128, ..., 1 whose plan a smaller window does not beat by
+                                  more than 1% in the planner's cost model, stopping at the first
+                                  plan without D2H spills (a window's first-level intermediates
+                                  are live together, so a tight budget needs a small window) */
   uint64_t seed;               /* tie-break RNG seed when deterministic == 0 */
   int32_t deterministic;       /* 1 (default) = lexicographic tie-breaks */
   int32_t keep_inputs_resident;/* 1 = node tensors uploaded by execute stay cached on the GPUs for
