@@ -54,7 +54,9 @@ def parse():
     ap.add_argument("--Lt", type=int, default=64)
     ap.add_argument("--rate", type=float, default=0.9)
     ap.add_argument("--dist", default="uniform", choices=["uniform", "gaussian"])
-    ap.add_argument("--policy", default="micco")
+    ap.add_argument("--policy", default="micco_affinity",
+                    help="scheduling policy (micco_affinity = MICCO's Alg. 1/2 with the last consumer's GPU "
+                         "preferred among Alg. 1's candidates; identical to micco on one GPU)")
     ap.add_argument("--window", type=int, default=0)
     ap.add_argument("--budget-gb", type=float, default=0.0,
                     help="per-GPU memory budget (0 = device free memory; c5 defaults to 25 GB: its "

@@ -72,12 +72,17 @@ typedef struct {
  * (PAPER.md L195-288); MICCO_NAIVE = bounds forced to (0,0,0) (L312);
  * ROUND_ROBIN = pair i of a vector to GPU i mod n; LEAST_LOADED = the GPU with
  * the least accumulated computation ("earliest available device", the Groute
- * rule of L312/L400). */
+ * rule of L312/L400); MICCO_AFFINITY = MICCO, except that when the GPU that last
+ * consumed the pair's first operand (else its second) is in Alg. 1's candidate queue,
+ * Alg. 2 takes it instead of the least-loaded candidate (not in the paper: once replicas
+ * of a tensor exist on several GPUs, least-computation alternates its consumers between
+ * them and spreads the replicas further; the candidate queue still bounds the imbalance). */
 enum {
   MICCO_POLICY_MICCO = 0,
   MICCO_POLICY_MICCO_NAIVE = 1,
   MICCO_POLICY_ROUND_ROBIN = 2,
-  MICCO_POLICY_LEAST_LOADED = 3
+  MICCO_POLICY_LEAST_LOADED = 3,
+  MICCO_POLICY_MICCO_AFFINITY = 4
 };
 
 typedef struct {

@@ -168,7 +168,7 @@ MICCO_API micco_status micco_create(micco_ctx **out, const micco_options *opt) {
     std::memcpy(&o, opt, std::min(opt->struct_size, sizeof(o)));
     o.struct_size = sizeof(o);
   }
-  if (o.policy < 0 || o.policy > 3 || o.window_graphs < 0 || o.mem_budget_bytes < 0 || o.dist_world < 0 ||
+  if (o.policy < 0 || o.policy > 4 || o.window_graphs < 0 || o.mem_budget_bytes < 0 || o.dist_world < 0 ||
       o.reorder < 0 || o.reorder > 1 || o.bound_model < 0 || o.bound_model > 2 ||
       (o.dist_world > 0 && (o.dist_rank < 0 || o.dist_rank >= o.dist_world)))
     return MICCO_ERR_ARG;

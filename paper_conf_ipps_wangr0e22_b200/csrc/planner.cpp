@@ -17,6 +17,7 @@
 #include <climits>
 #include <cmath>
 #include <limits>
+#include <cstdlib>
 #include <string>
 
 #include "core.h"
@@ -301,6 +302,8 @@ Plan make_plan(const Context &ctx, const PlanInput &in) {
       if (x >= 0 && x < NT && !((S.mask[x] >> g) & 1)) S.add_res(g, x);
 
   Scheduler sched(n, in.policy, in.reuse_bound, in.budget);
+  const bool affinity = in.policy == MICCO_POLICY_MICCO_AFFINITY;  // last consumer's GPU first
+  std::vector<int32_t> last_gpu(affinity ? NT : 0, -1);
   std::vector<std::vector<int32_t>> chunk(n);
   auto flush = [&](int g) {
     for (int32_t t : chunk[g]) S.emit(PlanOp::COMPUTE, g, -1, t);
@@ -334,8 +337,10 @@ Plan make_plan(const Context &ctx, const PlanInput &in) {
       p.b2 = same ? 0 : S.bytes(b);
       p.bout = (out.rank > 0 && y < 0) ? S.bytes(tk.out) : 0;
       p.flops = tk.flops + (y >= 0 ? ctx.tasks[plan.fused_dot[t]].flops : 0.0);
+      if (affinity) p.pref = last_gpu[a] >= 0 ? last_gpu[a] : (same ? -1 : last_gpu[b]);
       sched.mem = S.mem;
       const int g = sched.decide(p);
+      if (affinity) { last_gpu[a] = g; if (!same) last_gpu[b] = g; }
       const uint64_t bit = 1ULL << g;
       auto need_bytes = [&]() {
         int64_t need = p.bout;
@@ -448,7 +453,8 @@ Plan make_plan(const Context &ctx, const PlanInput &in) {
     plan.cache_hits = z.hits; plan.flops = z.flops;
   };
 
-  const bool per_stage = in.bound_mode != BOUNDS_FIXED && n > 1 && in.policy == MICCO_POLICY_MICCO;
+  const bool per_stage = in.bound_mode != BOUNDS_FIXED && n > 1 &&
+                         (in.policy == MICCO_POLICY_MICCO || in.policy == MICCO_POLICY_MICCO_AFFINITY);
   double predicted = 0;
   if (in.stream) in.stream->publish_fused(plan.fused_dot);
   for (int32_t s = 0; s < (int32_t)stages.size(); ++s) {

@@ -59,6 +59,9 @@ int Scheduler::assign(const SchedPair &p, uint64_t cand) const {
     int g = __builtin_ctzll(m);
     if (projected(g, p) > budget_[g]) evict = true;
   }
+  // MICCO_AFFINITY (p.pref >= 0 only under that policy): the last consumer's GPU, if Alg. 1
+  // admitted it and no oversubscription is projected
+  if (!evict && p.pref >= 0 && ((cand >> p.pref) & 1)) return p.pref;
   int best = -1;
   for (uint64_t m = cand; m; m &= m - 1) {
     int g = __builtin_ctzll(m);

@@ -21,6 +21,7 @@ struct SchedPair {
   bool same;                  // Tensor1 == Tensor2
   int64_t b1, b2, bout;       // bytes
   double flops;
+  int pref = -1;              // MICCO_AFFINITY: GPU of the operands' last consumer (-1 = none)
 };
 
 class Scheduler {

@@ -21,7 +21,7 @@ LIB_PATH = _HERE / "libmicco.so"
 MICCO_OK = 0
 STATUS_NAMES = {0: "OK", -1: "ERR_ARG", -2: "ERR_STATE", -3: "ERR_GRAPH", -4: "ERR_UNSUPPORTED",
                 -5: "ERR_OOM", -6: "ERR_CUDA", -7: "ERR_NCCL", -8: "ERR_RANGE"}
-POLICIES = {"micco": 0, "micco_naive": 1, "round_robin": 2, "least_loaded": 3}
+POLICIES = {"micco": 0, "micco_naive": 1, "round_robin": 2, "least_loaded": 3, "micco_affinity": 4}
 SYNTH_UNIFORM, SYNTH_INT3 = 0, 1
 
 

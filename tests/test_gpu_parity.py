@@ -125,8 +125,9 @@ def test_cross_run_invariance_bitwise():
     assert rel_err(ref, Co) <= TOL
     node_bytes = 24 * 24 * 4 * 16
     for n in (2, 3, 4, 8):
-        for pol in ("micco", "round_robin", "least_loaded", "micco_naive"):
-            C, _, _ = run_gpu(wl, n, [1, 2, 0] if pol == "micco" else None, policy=pol, window_graphs=16)
+        for pol in ("micco", "round_robin", "least_loaded", "micco_naive", "micco_affinity"):
+            C, _, _ = run_gpu(wl, n, [1, 2, 0] if pol.startswith("micco") and pol != "micco_naive" else None,
+                              policy=pol, window_graphs=16)
             assert np.array_equal(C, ref), (n, pol)
     for bd in ([0, 0, 0], [2, 2, 2], None):
         C, _, _ = run_gpu(wl, 4, bd)

@@ -290,3 +290,19 @@ def test_budget_sized_window():
     s256, _ = fixed.plan(1, [0, 0, 0])
     fixed.close()
     assert s0["n_stages"] == s256["n_stages"] and s0["bytes_h2d"] == s256["bytes_h2d"]
+
+
+def test_affinity_policy_cuts_peer_traffic():
+    """MICCO_AFFINITY (micco.h): on the weak-scaling workload (independent interleaved sets),
+    preferring the operands' last consumer among Alg. 1's candidates moves fewer bytes between
+    GPUs than plain MICCO, with the same balance guarantee (Alg. 1's candidate bound)."""
+    wl = workloads.c2_weak_sets(4, n_graphs=1000, N=8, Lt=2, rate=0.9, seed=2)
+    res = {}
+    for pol in ("micco", "micco_affinity"):
+        ctx = _ctx(mem_budget_bytes=1 << 30, policy=pol, window_graphs=256)
+        M.load_workload(ctx, wl)
+        res[pol], _ = ctx.plan(4, [1, 1, 1])
+        ctx.close()
+    assert res["micco_affinity"]["bytes_p2p"] < 0.7 * res["micco"]["bytes_p2p"]
+    assert res["micco_affinity"]["max_over_mean_load"] < 1.1
+    assert res["micco_affinity"]["n_gemm"] == res["micco"]["n_gemm"]

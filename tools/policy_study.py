@@ -30,7 +30,7 @@ sys.path.insert(0, str(ROOT))
 import paper_conf_ipps_wangr0e22_b200 as M  # noqa: E402
 from micco_inputs import workloads  # noqa: E402
 
-POLICIES = ["micco", "micco_naive", "round_robin", "least_loaded"]
+POLICIES = ["micco", "micco_affinity", "micco_naive", "round_robin", "least_loaded"]
 
 
 def plan(wl, policy, n_gpus, window, budget):

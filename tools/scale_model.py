@@ -30,8 +30,8 @@ import paper_conf_ipps_wangr0e22_b200 as M  # noqa: E402
 from micco_inputs import workloads  # noqa: E402
 
 
-def plan(wl, n, budget, warm):
-    ctx = M.Context(keep_inputs_resident=True, mem_budget_bytes=budget, dist_rank=0, dist_world=n)
+def plan(wl, n, budget, warm, policy):
+    ctx = M.Context(keep_inputs_resident=True, mem_budget_bytes=budget, dist_rank=0, dist_world=n, policy=policy)
     M.load_workload(ctx, wl)
     os.environ["MICCO_PLAN_WARM"] = "1" if warm else "0"
     try:
@@ -43,7 +43,7 @@ def plan(wl, n, budget, warm):
     finally:
         os.environ.pop("MICCO_PLAN_WARM", None)
         ctx.close()
-    return {"n_gpus": n, "warm": warm, "reuse_bound": bd, "model_s": pred,
+    return {"n_gpus": n, "warm": warm, "policy": policy, "reuse_bound": bd, "model_s": pred,
             "h2d_gb_per_gpu": st["bytes_h2d"] / n / 1e9, "d2h_gb_per_gpu": st["bytes_d2h"] / n / 1e9,
             "p2p_gb_per_gpu": st["bytes_p2p"] / n / 1e9, "evictions": st["evictions"],
             "max_over_mean_load": st["max_over_mean_load"], "host_plan_s": dt}
@@ -58,7 +58,7 @@ def main(argv=None):
     a = ap.parse_args(argv)
     budget = int(a.budget_gb * 1e9)
     rows = []
-    for kind in ("sets", "single"):
+    for kind, policy in (("sets", "micco_affinity"), ("sets", "micco"), ("single", "micco")):
         base = {}
         for n in [int(x) for x in a.gpus.split(",")]:
             if kind == "sets":
@@ -66,13 +66,13 @@ def main(argv=None):
             else:
                 wl = workloads.c2_meson_set(n_graphs=a.graphs * n, N=128, Lt=64, rate=0.9, seed=2)
             for warm in (False, True):
-                r = plan(wl, n, budget, warm)
+                r = plan(wl, n, budget, warm, policy)
                 r["workload"] = kind
                 if n == 1:
                     base[warm] = r["model_s"]
                 r["model_efficiency"] = base[warm] / r["model_s"] if warm in base else None
                 rows.append(r)
-                print(f"{kind:6s} n={n} {'warm' if warm else 'cold'}: model {r['model_s']:.3f} s "
+                print(f"{kind:6s} {policy:14s} n={n} {'warm' if warm else 'cold'}: model {r['model_s']:.3f} s "
                       f"(eff {r['model_efficiency'] or 0:.3f}), per GPU H2D {r['h2d_gb_per_gpu']:.1f} GB, "
                       f"P2P {r['p2p_gb_per_gpu']:.1f} GB, D2H {r['d2h_gb_per_gpu']:.1f} GB, "
                       f"evictions {r['evictions']}, load {r['max_over_mean_load']:.3f}", flush=True)
