@@ -93,7 +93,7 @@ typedef struct {
                                   agreed by an NCCL all-reduce, so every rank plans alike) */
   int32_t policy;              /* MICCO_POLICY_* */
   int32_t window_graphs;       /* graphs per window (one stream of vectors); 0 = auto: the largest
-                                  of 256, 128, ..., 1 whose plan a smaller window does not beat by
+                                  of 256·n_gpus, 128·n_gpus, ..., 1 whose plan a smaller window does not beat by
                                   more than 1% in the planner's cost model, stopping at the first
                                   plan without D2H spills (a window's first-level intermediates
                                   are live together, so a tight budget needs a small window) */

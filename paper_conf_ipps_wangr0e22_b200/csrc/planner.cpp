@@ -500,15 +500,19 @@ int32_t choose_window(const Context &ctx, PlanInput in) {
   // A window's stages are level-synchronous, so all the intermediates of its first level are
   // live at once: under a tight budget a large window spills what a smaller one would not
   // (C5 at 25 GB: W = 256 moves 178 GB over PCIe per execute, W = 128 0.4 GB).  Take the
-  // largest W in {256, 128, ..., 1} that a smaller W does not beat by more than 1% in the
+  // largest W in {256·n, 128·n, ..., 1} that a smaller W does not beat by more than 1% in the
   // cost model (which prices host bytes); stop at the first plan that spills nothing (a smaller
   // window only bounds the live set of intermediates).  Stages stay as large as the
   // budget allows (fewer, larger grouped launches).
   in.stream = nullptr;
-  int32_t best_w = 256;
+  // The first candidate is 256 graphs per GPU: a stage then gives each GPU as many pairs as a
+  // one-GPU stage (grouped launches of the same size; an 8-GPU weak-scaling plan has 81
+  // instead of 628 stages).
+  const int32_t w0 = 256 * std::max(1, in.n_gpus);
+  int32_t best_w = w0;
   double best = 0;
   bool have = false;
-  for (int32_t W = 256; W >= 1; W /= 2) {
+  for (int32_t W = w0; W >= 1; W /= 2) {
     in.window_graphs = W;
     const Plan p = make_plan(ctx, in);
     if (!have || p.predicted_s < best * 0.99) {
