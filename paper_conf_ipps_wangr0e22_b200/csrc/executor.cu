@@ -203,12 +203,20 @@ struct Executor::Impl {
     for (auto &d : devs) {
       if (d.dev < 0) continue;
       cudaSetDevice(d.dev);
+      if (d.init) {  // hand the pool's cached blocks back, so the next setup's budget (from the
+        cudaMemPool_t pool;  // device's free memory) does not count them as used
+        if (cudaDeviceGetDefaultMemPool(&pool, d.dev) == cudaSuccess) {
+          cudaDeviceSynchronize();
+          cudaMemPoolTrimTo(pool, 0);
+        }
+      }
       if (d.scalars) cudaFree(d.scalars);
       d.scalars = nullptr;
       d.sync_events.destroy();
       d.timing_events.destroy();
     }
     if (d_vals) { cudaSetDevice(vals_dev); cudaFree(d_vals); d_vals = nullptr; }
+    vals_elems = 0;  // (a re-setup for another GPU count must reallocate the value table)
     if (h_corr) { cudaFreeHost(h_corr); h_corr = nullptr; }
     if (comm && nccl().ok) nccl().CommDestroy(comm);
     comm = nullptr;

@@ -297,3 +297,21 @@ def test_streamed_planning_bitwise(monkeypatch):
         for a, b in zip(res["0"], res["1"]):
             assert np.array_equal(a, b), n
         assert rel_err(res["0"][-1], Co) <= TOL
+
+
+def test_gpu_count_change_in_one_context():
+    """One context executed on 2, then 1, then 3 logical GPUs (each switch tears the executor
+    down and sets it up again): the same C(t) bit for bit, and graph values readable after
+    each.  (Regression: the per-graph value table was not reallocated after a re-setup.)"""
+    wl = workloads.c2_meson_set(n_graphs=90, N=24, Lt=3, rate=0.7)
+    ctx = M.Context(keep_inputs_resident=True)
+    M.load_workload(ctx, wl)
+    out = []
+    for n in (2, 1, 3, 1):
+        ctx.execute(n)
+        out.append(ctx.correlator())
+        assert np.isfinite(ctx.graph_value(len(wl.graphs) - 1, 2))
+    ctx.close()
+    for C in out[1:]:
+        assert np.array_equal(C, out[0])
+    assert rel_err(out[0], oracle.correlator(wl)) <= TOL
