@@ -24,3 +24,30 @@ for n in (2, 1):
 ctx.close()
 print("bitwise equal n=1 vs n=2:", bool(np.array_equal(res[1], res[2])))
 assert np.array_equal(res[1], res[2])
+
+
+def scenario(name, wl, ns, **kw):
+    """C(t) of wl on each logical GPU count in ns, one fresh context per count: bitwise equal."""
+    ref = None
+    for n in ns:
+        c = M.Context(**kw)
+        M.load_workload(c, wl)
+        t = time.perf_counter()
+        c.execute(n)
+        dt = time.perf_counter() - t
+        st = c.stats()
+        C = c.correlator()
+        c.close()
+        print(f"{name} n={n}: {dt*1e3:.0f} ms, p2p {st['bytes_p2p']/1e9:.1f} GB, h2d {st['bytes_h2d']/1e9:.1f} GB, "
+              f"d2h {st['bytes_d2h']/1e9:.1f} GB, evictions {st['evictions']}", flush=True)
+        if ref is None:
+            ref = C
+        assert np.array_equal(C, ref), (name, n)
+    print(f"{name}: bitwise equal over {ns}")
+
+
+scenario("c5 25GB", workloads.c5_mixed(n_combos=1, Nb=64, Nm=256, Lt=16, pool=2, meson_graphs=64),
+         (1, 2, 4), mem_budget_bytes=int(25e9), policy="micco_affinity")
+scenario("c5 25GB W=256", workloads.c5_mixed(n_combos=1, Nb=64, Nm=256, Lt=16, pool=2, meson_graphs=64),
+         (1, 2), mem_budget_bytes=int(25e9), window_graphs=256)
+scenario("c4", workloads.c4_two_baryon(n_combos=8, N=64, Lt=64, order="greedy"), (1, 3), policy="micco_affinity")
