@@ -257,14 +257,23 @@ void build_graph(Context &ctx, int32_t n_inst, const int64_t *node_ids, int32_t 
       if (st.cb >= 0) {  // the kernels must be able to read both operands in place
         const Comp &A = comps[st.ca], &B = comps[st.cb];
         bool ok;
+        const long long lim = (1LL << 31) - 1;  // the kernels keep per-slice offsets in 32 bits
+        bool fits = true;
         if (rr > 0) {
           GemmLayout gl;
           ok = gemm_layout(A.rank, A.dim, B.rank, B.dim, st.c, st.pa, st.pb, gl);
+          // (the executor's limits, checked here so a graph the kernels cannot run is refused
+          // at add_graph, not part-way through an execute; 64 × 32 is the smallest tile)
+          if (ok)
+            fits = gl.sliceA <= lim && gl.sliceB <= lim && gl.sliceC <= lim &&
+                   (long long)ctx.Lt * gl.Mo * gl.No * ((gl.Mi + 63) / 64) * ((gl.Ni + 31) / 32) < (1LL << 32);
         } else {
           DotLayout dl;
           ok = dot_layout(A.rank, A.dim, B.rank, B.dim, st.c, st.pa, st.pb, dl);
+          if (ok) fits = dl.sliceA <= lim && dl.sliceB <= lim;
         }
         if (!ok) fail(MICCO_ERR_UNSUPPORTED, "add_graph: contraction layout not supported by the kernels");
+        if (!fits) fail(MICCO_ERR_UNSUPPORTED, "add_graph: a tensor slice exceeds 2^31 elements (kernel limit)");
       }
       if (!commit) chosen.push_back(e);
       // mark contracted edges done

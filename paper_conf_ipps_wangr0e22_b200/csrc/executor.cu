@@ -156,6 +156,9 @@ struct LGpu {
   std::vector<DotDesc> dot;
   std::vector<double2 *> part_allocs;  // fused-dot partials of the pending batch
   long long gemm_tiles = 0, dot_ctas = 0;
+  // bytes the H2D prefetch may run ahead of the compute stream: the device memory left outside
+  // the planned budgets, shared by the logical GPUs on this device (budgets())
+  int64_t prefetch_cap = kPrefetchBytes;
 };
 
 }  // namespace
@@ -291,6 +294,25 @@ struct Executor::Impl {
       CK(cudaStreamCreateWithFlags(&l.cst, cudaStreamNonBlocking));
       CK(cudaStreamCreateWithFlags(&l.pst, cudaStreamNonBlocking));
     }
+    // Peer access to stream-ordered pool memory is granted per pool (cudaDeviceEnablePeerAccess
+    // covers cudaMalloc memory only): every device in use may read every other's pool, so a
+    // peer copy of a replica is a direct NVLink transfer.
+    for (int d = 0; d < ndev; ++d) {
+      if (!devs[d].init) continue;
+      cudaMemPool_t pool;
+      CK(cudaDeviceGetDefaultMemPool(&pool, d));
+      for (int p = 0; p < ndev; ++p) {
+        if (p == d || !devs[p].init) continue;
+        int can = 0;
+        cudaDeviceCanAccessPeer(&can, p, d);
+        if (!can) continue;
+        cudaMemAccessDesc acc{};
+        acc.location.type = cudaMemLocationTypeDevice;
+        acc.location.id = p;
+        acc.flags = cudaMemAccessFlagsProtReadWrite;
+        CK(cudaMemPoolSetAccess(pool, &acc, 1));
+      }
+    }
     if (dist()) {
       if (!c.have_nccl_id) fail(MICCO_ERR_STATE, "multi-process mode needs micco_set_nccl_id before execute");
       if (!nccl().ok) fail(MICCO_ERR_NCCL, "NCCL unavailable: " + nccl().why);
@@ -308,7 +330,6 @@ struct Executor::Impl {
     std::vector<int> per_dev(ndev, 0);
     for (int i = 0; i < n; ++i) per_dev[g[i].dev]++;
     for (int i = 0; i < n; ++i) {
-      if (c.opt.mem_budget_bytes > 0) { b[i] = c.opt.mem_budget_bytes; continue; }
       size_t fr = 0, tot = 0;
       if (g[i].local || !dist()) {
         CK(cudaSetDevice(g[i].dev));
@@ -318,9 +339,19 @@ struct Executor::Impl {
         CK(cudaSetDevice(g[my_rank()].dev));
         CK(cudaMemGetInfo(&fr, &tot));
       }
-      int k = dist() ? 1 : per_dev[g[i].dev];
-      int64_t usable = (int64_t)(fr * 0.92) - (2LL << 30);
-      b[i] = std::max<int64_t>(usable / k, 1LL << 28);
+      const int k = dist() ? 1 : per_dev[g[i].dev];
+      if (c.opt.mem_budget_bytes > 0) {
+        b[i] = c.opt.mem_budget_bytes;
+      } else {
+        int64_t usable = (int64_t)(fr * 0.92) - (2LL << 30);
+        b[i] = std::max<int64_t>(usable / k, 1LL << 28);
+      }
+      // The prefetch (and peer look-ahead) allocate beyond what the plan has freed so far:
+      // keep them inside the memory the budgets leave free on this device, minus a reserve
+      // for the fused-dot partials and the allocator's rounding (with several
+      // logical GPUs per device or a caller budget near capacity the pool could run out).
+      const int64_t slack = ((int64_t)fr - k * b[i] - (1LL << 30)) / k;
+      g[i].prefetch_cap = std::min<int64_t>(kPrefetchBytes, std::max<int64_t>(slack, 0));
     }
     if (dist()) {  // every rank must plan with identical budgets: the minimum over ranks
       int64_t mn = *std::min_element(b.begin(), b.end());
@@ -544,14 +575,14 @@ struct Executor::Impl {
       case PlanOp::H2D: {
         // Prefetch on the copy stream (NEXT #1 of SURVEY.md §8(f); "asynchronous
         // data copy and prefetching"): the copy for chunk k+1 may start once chunk k-1 has
-        // finished (bounded look-ahead keeps the pool within the planned budget + one chunk);
+        // finished (bounded look-ahead: at most prefetch_cap bytes beyond the planned budget);
         // the compute stream waits for the copy right away, so everything it enqueues later
         // (kernels, peer reads) sees the data, while already-enqueued kernels keep running.
         LGpu &l = g[op.gpu];
         if (!l.local) return;
         CK(cudaSetDevice(l.dev));
         // look-ahead: the copy for stage s may run while stages s-1 .. s-kLookahead compute;
-        // bounded by bytes so the pool stays within the budget's slack (0.08 × free + 2 GiB)
+        // bounded by bytes so the pool stays within the device memory the budgets leave free
         {
           const int64_t nb = bytes_of(op.id);
           l.fetch_bytes_since.push_back(nb);
@@ -561,7 +592,7 @@ struct Executor::Impl {
           // walk back over flushed chunks while the prefetch window stays small
           while (depth < kLookahead && depth < (int)nf) {
             ahead += l.chunk_fetch[nf - 1 - depth];
-            if (ahead > kPrefetchBytes) break;
+            if (ahead > l.prefetch_cap) break;
             ++depth;
           }
           if ((int)nf > depth) CK(cudaStreamWaitEvent(l.cst, l.flush_ev[nf - 1 - depth], 0));
@@ -676,7 +707,47 @@ struct Executor::Impl {
 
   // ---------------------------------------------------------------- execute
 
+  // Any failure inside an execute (a CUDA error, a planner exception rethrown mid-replay)
+  // leaves per-GPU state that the next execute must not see: pending descriptors whose
+  // output pointers may point into a freed table, replicas the cache bookkeeping no longer
+  // matches.  Drain the streams and drop all of it, then rethrow.
   void execute(int n_gpus, const int32_t *bd) {
+    try {
+      execute_impl(n_gpus, bd);
+    } catch (...) {
+      recover();
+      throw;
+    }
+  }
+
+  void recover() noexcept {
+    for (auto &l : g) {
+      if (!l.local || !l.st) continue;
+      cudaSetDevice(l.dev);
+      cudaStreamSynchronize(l.st);
+      if (l.cst) cudaStreamSynchronize(l.cst);
+      if (l.pst) cudaStreamSynchronize(l.pst);
+      for (auto &p : l.ptr)
+        if (p) { cudaFree(p); p = nullptr; }
+      for (double2 *p : l.part_allocs) cudaFree(p);
+      l.part_allocs.clear();
+      l.gemm.clear();
+      l.dot.clear();
+      l.readers.clear();
+      l.flush_ev.clear();
+      l.chunk_fetch.clear();
+      l.fetch_bytes_since.clear();
+      l.pending_fetch = 0;
+    }
+    cudaGetLastError();  // (a non-sticky error must not leak into the next call)
+    cached_nodes.clear();
+    stream_ok_n = 0;
+    spill_host.clear();
+    spill_ev.clear();
+    spill_arena.rewind();
+  }
+
+  void execute_impl(int n_gpus, const int32_t *bd) {
     auto t0 = std::chrono::steady_clock::now();
     setup(n_gpus);
     for (auto &l : g)

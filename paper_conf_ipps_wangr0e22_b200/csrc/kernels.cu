@@ -1069,9 +1069,15 @@ int gemm_kernel_class(int layout_cls, int Ko) {
 bool gemm_fused_dot_ok() { return gemm_variant() != 1; }
 
 cudaError_t launch_gemm_group(const GemmBatch *b, long long total_tiles, int cls, cudaStream_t st) {
-  static bool attr_set = false;  // per process; the attribute is per-function, all devices
+  // (one host thread launches: the executor replays the plan sequentially)
+  // The shared-memory opt-in is recorded per device context: track it per device, so the
+  // persistent GEMMs on a second (third, ...) device of one process get it too.
+  static unsigned long long attr_set = 0;  // bit d: set on device d
   const int variant = gemm_variant();
-  if (!attr_set) {
+  int cur_dev = 0;
+  if (cudaError_t e = cudaGetDevice(&cur_dev); e != cudaSuccess) return e;
+  const unsigned long long dev_bit = 1ull << (cur_dev & 63);
+  if (!(attr_set & dev_bit)) {
     cudaError_t e = cudaFuncSetAttribute(zgemm_dmma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, GEMM_SMEM);
     if (e != cudaSuccess) return e;
     for (int c = 0; c < 4; ++c) {
@@ -1093,12 +1099,11 @@ cudaError_t launch_gemm_group(const GemmBatch *b, long long total_tiles, int cls
         if (e != cudaSuccess) return e;
       }
     }
-    attr_set = true;
+    attr_set |= dev_bit;
   }
   if (total_tiles <= 0) return cudaSuccess;
-  int dev = 0, sms = 148;
-  cudaGetDevice(&dev);
-  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  int sms = 148;
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, cur_dev);
   if (variant == 1 || cls == 4) {  // per-tile kernel; the only one that gathers strided operands
     long long grid = total_tiles < (1LL << 30) ? total_tiles : (1LL << 30);
     zgemm_dmma_kernel<<<(unsigned)grid, NT, GEMM_SMEM, st>>>(*b, total_tiles);

@@ -337,6 +337,7 @@ Plan make_plan(const Context &ctx, const PlanInput &in) {
       p.b2 = same ? 0 : S.bytes(b);
       p.bout = (out.rank > 0 && y < 0) ? S.bytes(tk.out) : 0;
       p.flops = tk.flops + (y >= 0 ? ctx.tasks[plan.fused_dot[t]].flops : 0.0);
+      if (has_y) { p.m3 = S.mask[y]; p.b3 = S.bytes(y); }
       if (affinity) p.pref = last_gpu[a] >= 0 ? last_gpu[a] : (same ? -1 : last_gpu[b]);
       sched.mem = S.mem;
       const int g = sched.decide(p);

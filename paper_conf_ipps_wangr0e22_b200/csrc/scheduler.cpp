@@ -50,6 +50,7 @@ int64_t Scheduler::projected(int g, const SchedPair &p) const {  // reading #16
   int64_t m = mem[g];
   if (!((p.m1 >> g) & 1)) m += p.b1;
   if (!p.same && !((p.m2 >> g) & 1)) m += p.b2;
+  if (p.b3 > 0 && !((p.m3 >> g) & 1)) m += p.b3;  // (the planner's need_bytes counts it too)
   return m + p.bout;
 }
 
@@ -69,7 +70,8 @@ int Scheduler::assign(const SchedPair &p, uint64_t cand) const {
     if (!evict) {  // lines 6-11: least computation, ties least memory, then id (#17)
       if (com_[g] < com_[best] || (com_[g] == com_[best] && mem[g] < mem[best])) best = g;
     } else {       // lines 12-17: most available memory, ties least computation, then id
-      if (mem[g] < mem[best] || (mem[g] == mem[best] && com_[g] < com_[best])) best = g;
+      const int64_t fg = budget_[g] - mem[g], fb = budget_[best] - mem[best];
+      if (fg > fb || (fg == fb && com_[g] < com_[best])) best = g;
     }
   }
   return best;                                             // line 18

@@ -20,6 +20,8 @@ struct SchedPair {
   uint64_t m1, m2;            // residency masks of Tensor1, Tensor2 (bit g = resident on GPU g)
   bool same;                  // Tensor1 == Tensor2
   int64_t b1, b2, bout;       // bytes
+  uint64_t m3 = 0;            // a third operand read by the task (the fused final dot's partner)
+  int64_t b3 = 0;             // ... and its bytes (0 = none)
   double flops;
   int pref = -1;              // MICCO_AFFINITY: GPU of the operands' last consumer (-1 = none)
 };

@@ -91,7 +91,8 @@ def build_lib(force: bool = False, jobs: int = 8) -> Path:
             _drain(procs)
     _drain(procs)
     tmp = LIB_SO.with_suffix(".so.tmp")
-    _run([nvcc] + NVCC_ARCH + ["-shared", "-o", tmp] + objs + ["-lpthread", "-ldl"])
+    # shared cudart: the library links the system libcudart.so instead of embedding a static copy
+    _run([nvcc] + NVCC_ARCH + ["-shared", "-cudart", "shared", "-o", tmp] + objs + ["-lpthread", "-ldl"])
     os.replace(tmp, LIB_SO)
     return LIB_SO
 
