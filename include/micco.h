@@ -117,6 +117,11 @@ typedef struct {
                                   fitted regression (a random forest over vector
                                   features, trained offline on mode-1 choices by
                                   tools/train_bounds.py) */
+  int32_t scalar_tables;       /* where rank-0 results (per-slice scalars) are written before the
+                                  final cross-GPU reduce: 0 (default) one table per CUDA device;
+                                  1 one table per logical GPU, so the combine (peer copy + exact
+                                  accumulate, every slot nonzero in one table only) runs even when
+                                  several logical GPUs share a device.  C(t) is bitwise the same */
 } micco_options;
 
 /* Fill *opt with the defaults (struct_size set). */
@@ -211,12 +216,25 @@ typedef struct {
   int32_t gemm_3m;             /* 1 if the GEMMs used 3 real DMMA products per complex MAC (Gauss) */
   double gemm_dmma_flops;      /* flops actually executed on the DMMA pipe by the GEMMs
                                   (= gemm_flops, or 6/8 of it with the 3M scheme) */
+  double dot_main_ms;          /* device time of the standalone dot launches (flat and transposed
+                                  dots of two tensors; not traces, not fused-dot partial sums) */
+  double dot_main_bytes;       /* algorithmic bytes those dots read: 16 B per element of both
+                                  operands, all Lt slices (the HBM roofline numerator) */
+  int64_t dot_main_launches;
+  double plan_ms;              /* host time of make_plan for this execute (overlapped with the
+                                  replay when planning streams; sched_ms = the same) */
 } micco_stats;
 
 MICCO_API micco_status micco_get_stats(const micco_ctx *ctx, micco_stats *out);
 
 /* Drop every cached replica (inputs kept by keep_inputs_resident). */
 MICCO_API micco_status micco_release_cache(micco_ctx *ctx);
+
+/* Switch the scheduling policy (MICCO_POLICY_*) of an existing context, for policy comparisons
+ * on one loaded graph set (§V-B).  Drops cached replicas, so the next
+ * execute starts cold; bounds chosen by an earlier sweep are re-chosen for the new policy.
+ * Multi-process mode: every rank must make the same call. */
+MICCO_API micco_status micco_set_policy(micco_ctx *ctx, int32_t policy);
 
 /* ---- multi-process mode (one process per GPU; torch.distributed is the plumbing) ----
  * Rank 0 calls micco_nccl_unique_id, broadcasts the 128 bytes, then every rank calls
@@ -226,6 +244,16 @@ MICCO_API micco_status micco_release_cache(micco_ctx *ctx);
  * combining the per-graph scalars with one ncclAllReduce. */
 MICCO_API micco_status micco_nccl_unique_id(uint8_t out[128]);
 MICCO_API micco_status micco_set_nccl_id(micco_ctx *ctx, const uint8_t id[128]);
+
+/* ---- device probe (measurement tooling, not the paper's interface) ----
+ * The FP64 tensor-pipe ceiling of the current CUDA device: a register-only loop of
+ * mma.sync m8n8k4 f64 (SASS DMMA.8x8x4), 16 warps per SM on every SM, 8 independent
+ * accumulator chains per warp, for about `seconds` of device time (one short burst launch
+ * first, then back-to-back launches).  *burst_tflops = the best single launch,
+ * *sustained_tflops = the whole run (bench.py's roofline denominator for kernels timed
+ * inside a long step; MEASURED_PEAKS.json has no FP64 figure).  512 flops per DMMA. */
+MICCO_API micco_status micco_probe_fp64_peak(double seconds, double *burst_tflops,
+                                             double *sustained_tflops);
 
 /* ---- introspection for host-side tests (no GPU needed) ---- */
 

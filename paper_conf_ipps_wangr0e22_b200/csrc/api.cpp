@@ -12,6 +12,7 @@
 
 #include "core.h"
 #include "executor.h"
+#include "kernels.h"
 #include "micco_inputs/synth.h"
 #include "scheduler.h"
 
@@ -170,6 +171,7 @@ MICCO_API micco_status micco_create(micco_ctx **out, const micco_options *opt) {
   }
   if (o.policy < 0 || o.policy > 4 || o.window_graphs < 0 || o.mem_budget_bytes < 0 || o.dist_world < 0 ||
       o.reorder < 0 || o.reorder > 1 || o.bound_model < 0 || o.bound_model > 2 ||
+      o.scalar_tables < 0 || o.scalar_tables > 1 ||
       (o.dist_world > 0 && (o.dist_rank < 0 || o.dist_rank >= o.dist_world)))
     return MICCO_ERR_ARG;
   micco_ctx *c = new (std::nothrow) micco_ctx;
@@ -476,9 +478,24 @@ MICCO_API micco_status micco_get_stats(const micco_ctx *ctx, micco_stats *out) {
   return MICCO_OK;
 }
 
+MICCO_API micco_status micco_probe_fp64_peak(double seconds, double *burst_tflops, double *sustained_tflops) {
+  if (!burst_tflops || !sustained_tflops || !(seconds >= 0)) return MICCO_ERR_ARG;
+  int n = 0;
+  if (cudaGetDeviceCount(&n) != cudaSuccess || n < 1) return MICCO_ERR_CUDA;
+  return micco::probe_fp64_peak(seconds, burst_tflops, sustained_tflops) == cudaSuccess ? MICCO_OK : MICCO_ERR_CUDA;
+}
+
 MICCO_API micco_status micco_release_cache(micco_ctx *ctx) {
   return guard(ctx, [&] {
     if (ctx->c.exec) ctx->c.exec->release_cache();
+  });
+}
+
+MICCO_API micco_status micco_set_policy(micco_ctx *ctx, int32_t policy) {
+  return guard(ctx, [&] {
+    if (policy < 0 || policy > 4) fail(MICCO_ERR_ARG, "unknown policy");
+    if (ctx->c.exec) ctx->c.exec->release_cache();
+    ctx->c.opt.policy = policy;
   });
 }
 

@@ -128,15 +128,22 @@ struct EventPool {
 
 struct DevState {
   int dev = -1;
-  double2 *scalars = nullptr;
-  size_t scalar_elems = 0;
   EventPool sync_events, timing_events;
   bool init = false;
 };
 
+// A scalar table [slot][t] (rank-0 results).  One per device by default; one per logical GPU
+// with options.scalar_tables = 1, so that the cross-GPU combine (peer copy + exact
+// accumulate) also runs when several logical GPUs share one device.
+struct ScalarTable {
+  int dev = -1;
+  double2 *p = nullptr;
+  size_t elems = 0;
+};
+
 struct Timed {
   cudaEvent_t a, b;
-  int kind;  // 0 gemm, 1 dot, 2 copy
+  int kind;  // 0 gemm, 1 dot (warp kernel: traces, fused-dot sums), 2 copy, 3 dot (CTA kernel)
   int dev;
 };
 
@@ -169,6 +176,7 @@ struct Executor::Impl {
   int n = 0;  // logical GPUs
   std::vector<LGpu> g;
   std::vector<DevState> devs;
+  std::vector<ScalarTable> tables;  // indexed by table_of(logical GPU)
   std::vector<Timed> timed;
   std::unordered_map<int32_t, double *> spill_host;
   std::unordered_map<int32_t, std::pair<int, cudaEvent_t>> spill_ev;
@@ -194,6 +202,10 @@ struct Executor::Impl {
   double2 *h_corr = nullptr;
   int64_t launches = 0;
   bool dist() const { return c.opt.dist_world > 0; }
+  int table_of(int i) const { return c.opt.scalar_tables ? i : g[i].dev; }
+  double2 *table_row(const LGpu &l, int32_t slot) const {
+    return tables[table_of(l.idx)].p + (size_t)slot * c.Lt;
+  }
   int my_rank() const { return c.opt.dist_rank; }
 
   explicit Impl(Context &ctx) : c(ctx) {}
@@ -213,11 +225,12 @@ struct Executor::Impl {
           cudaMemPoolTrimTo(pool, 0);
         }
       }
-      if (d.scalars) cudaFree(d.scalars);
-      d.scalars = nullptr;
       d.sync_events.destroy();
       d.timing_events.destroy();
     }
+    for (auto &t : tables)
+      if (t.p) { cudaSetDevice(t.dev); cudaFree(t.p); }
+    tables.clear();
     if (d_vals) { cudaSetDevice(vals_dev); cudaFree(d_vals); d_vals = nullptr; }
     vals_elems = 0;  // (a re-setup for another GPU count must reallocate the value table)
     if (h_corr) { cudaFreeHost(h_corr); h_corr = nullptr; }
@@ -464,7 +477,7 @@ struct Executor::Impl {
       for (const DotDesc &d : l.dot) by[dot_class(d.mode)].push_back(d);
       l.dot.clear();
       for (int c = 0; c < 2; ++c) {
-        launch_batch(l, by[c], 1, c, *dot_batch, kDotBatch, [](DotDesc *d, int cnt) {
+        launch_batch(l, by[c], c == 0 ? 1 : 3, c, *dot_batch, kDotBatch, [](DotDesc *d, int cnt) {
           long long acc = 0;
           for (int i = 0; i < cnt; ++i) {
             d[i].cta_begin = acc;
@@ -531,7 +544,7 @@ struct Executor::Impl {
         l.part_allocs.push_back(d.part);
         DotDesc r{};
         r.A = d.part; r.B = nullptr;
-        r.out = devs[l.dev].scalars + (size_t)c.tensors[dk.out].scalar_slot * c.Lt;
+        r.out = table_row(l, c.tensors[dk.out].scalar_slot);
         r.sAt = tps; r.mode = 3; r.X = (int)tps; r.Lt = c.Lt;
         for (int i = 0; i < 3; ++i) r.O[i] = 1;
         l.dot.push_back(r);
@@ -559,7 +572,7 @@ struct Executor::Impl {
         fail(MICCO_ERR_UNSUPPORTED, "executor: tensor slice exceeds 2^31 elements");
       DotDesc d{};
       d.A = pa; d.B = pb;
-      d.out = devs[l.dev].scalars + (size_t)c.tensors[tk.out].scalar_slot * c.Lt;
+      d.out = table_row(l, c.tensors[tk.out].scalar_slot);
       d.sAt = L.sliceA; d.sBt = L.sliceB;
       d.mode = L.mode; d.nO = L.nO; d.X = L.X; d.Y = L.Y;
       d.sAx = L.sAx; d.sAy = L.sAy; d.sBx = L.sBx; d.sBy = L.sBy;
@@ -567,6 +580,7 @@ struct Executor::Impl {
       d.Lt = c.Lt;
       l.dot.push_back(d);
       st.dot_bytes += (double)(L.sliceA + L.sliceB) * 16.0 * c.Lt;
+      if (dot_class(L.mode) == 1) st.dot_main_bytes += (double)(L.sliceA + L.sliceB) * 16.0 * c.Lt;
     }
   }
 
@@ -789,7 +803,7 @@ struct Executor::Impl {
     Plan plan;
     bool sweep = false;  // whole-plan bound sweep (27 plans): synchronous
     // choices cached across executes are valid for this GPU count and this DAG
-    const int64_t dag_key = (int64_t)c.tasks.size() * 1000003 + (int64_t)c.graphs.size();
+    const int64_t dag_key = ((int64_t)c.tasks.size() * 1000003 + (int64_t)c.graphs.size()) * 8 + c.opt.policy;
     if (dag_key != cache_dag_key) {
       chosen_bd_n = chosen_w_n = 0;
       cache_dag_key = dag_key;
@@ -861,28 +875,30 @@ struct Executor::Impl {
 
     micco_stats st{};
     st.struct_size = sizeof(st);
-    // scalar tables (one per device in use), zeroed before any dot writes
+    // scalar tables (one per device in use, or one per logical GPU), zeroed before any dot
+    // writes; every logical GPU writing a table waits for its zeroing
     const size_t selems = (size_t)std::max(1, c.n_scalar_slots) * c.Lt;
-    std::vector<int> first_lgpu(ndev, -1);
+    const int ntab = c.opt.scalar_tables ? n : ndev;
+    if ((int)tables.size() < ntab) tables.resize(ntab);
+    std::vector<int> first_lgpu(ntab, -1);  // the logical GPU that zeroes (and owns) table k
     for (int i = 0; i < n; ++i)
-      if (g[i].local && first_lgpu[g[i].dev] < 0) first_lgpu[g[i].dev] = i;
-    for (int d = 0; d < ndev; ++d) {
-      if (first_lgpu[d] < 0) continue;
-      LGpu &l = g[first_lgpu[d]];
-      CK(cudaSetDevice(d));
-      if (devs[d].scalar_elems < selems) {
+      if (g[i].local && first_lgpu[table_of(i)] < 0) first_lgpu[table_of(i)] = i;
+    for (int k = 0; k < ntab; ++k) {
+      if (first_lgpu[k] < 0) continue;
+      LGpu &l = g[first_lgpu[k]];
+      ScalarTable &T = tables[k];
+      CK(cudaSetDevice(l.dev));
+      if (T.elems < selems || T.dev != l.dev) {
         CK(cudaStreamSynchronize(l.st));
-        if (devs[d].scalars) CK(cudaFree(devs[d].scalars));
-        CK(cudaMalloc((void **)&devs[d].scalars, selems * sizeof(double2)));
-        devs[d].scalar_elems = selems;
+        if (T.p) { CK(cudaSetDevice(T.dev)); CK(cudaFree(T.p)); CK(cudaSetDevice(l.dev)); }
+        CK(cudaMalloc((void **)&T.p, selems * sizeof(double2)));
+        T.elems = selems;
+        T.dev = l.dev;
       }
-      CK(cudaMemsetAsync(devs[d].scalars, 0, selems * sizeof(double2), l.st));
-      cudaEvent_t e = record(first_lgpu[d]);
+      CK(cudaMemsetAsync(T.p, 0, selems * sizeof(double2), l.st));
+      cudaEvent_t e = record(first_lgpu[k]);
       for (int i = 0; i < n; ++i)
-        if (g[i].local && g[i].dev == d && i != first_lgpu[d]) {
-          CK(cudaSetDevice(d));
-          CK(cudaStreamWaitEvent(g[i].st, e, 0));
-        }
+        if (g[i].local && table_of(i) == k && i != first_lgpu[k]) CK(cudaStreamWaitEvent(g[i].st, e, 0));
     }
     auto tq0 = std::chrono::steady_clock::now();
     if (streaming) {
@@ -935,17 +951,25 @@ struct Executor::Impl {
     CK(cudaSetDevice(H.dev));
     for (int i = 0; i < n; ++i)
       if (i != home && g[i].local) CK(cudaStreamWaitEvent(H.st, record(i), 0));
-    double2 *S = devs[H.dev].scalars;
+    double2 *S = tables[table_of(home)].p;
     if (dist()) {
       // every NCCL call of this rank in one order: the all-reduce after the last send/recv
       if (H.pst) CK(cudaStreamWaitEvent(H.st, record_on(home, H.pst), 0));
       NK(nccl().AllReduce(S, S, selems * 2, ncclDouble, ncclSum, comm, H.st));
     } else {
-      for (int d = 0; d < ndev; ++d) {
-        if (d == H.dev || first_lgpu[d] < 0) continue;
+      // Exact combine: every slot is nonzero in exactly one table (the producing GPU's), so
+      // S += T adds zeros everywhere else, and the result is bitwise independent of the GPU
+      // count and of the order of the tables (north_star: final cross-GPU reduce).
+      for (int k = 0; k < ntab; ++k) {
+        if (k == table_of(home) || first_lgpu[k] < 0) continue;
+        const ScalarTable &T = tables[k];
         double2 *tmp = alloc(H, (int64_t)(selems * sizeof(double2)));
-        CK(cudaMemcpyPeerAsync(tmp, H.dev, devs[d].scalars, d, selems * sizeof(double2), H.st));
+        if (T.dev == H.dev)
+          CK(cudaMemcpyAsync(tmp, T.p, selems * sizeof(double2), cudaMemcpyDeviceToDevice, H.st));
+        else
+          CK(cudaMemcpyPeerAsync(tmp, H.dev, T.p, T.dev, selems * sizeof(double2), H.st));
         CK(launch_accumulate(S, tmp, (long long)selems, H.st));
+        ++launches;
         CK(cudaFreeAsync(tmp, H.st));
       }
     }
@@ -1008,9 +1032,16 @@ struct Executor::Impl {
       st.kernel_ms += ms;
       if (tm.kind == 0) { st.gemm_kernel_ms += ms; ++st.gemm_launches; }
       else if (tm.kind == 1) { st.dot_kernel_ms += ms; ++st.dot_launches; }
+      else if (tm.kind == 3) {
+        st.dot_kernel_ms += ms;
+        ++st.dot_launches;
+        st.dot_main_ms += ms;
+        ++st.dot_main_launches;
+      }
     }
     st.wall_ms = std::chrono::duration<double, std::milli>(t2 - t0).count();
     st.sched_ms = plan_ms;  // planning time (overlapped with the replay when streamed)
+    st.plan_ms = plan_ms;
     stream_ok_n = n;
     st.evictions = plan.evictions;
     st.cache_hits = plan.cache_hits;

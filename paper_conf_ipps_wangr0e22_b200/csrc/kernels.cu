@@ -11,6 +11,7 @@
 //   Cr += Ar·Br + (−Ai)·Bi,   Ci += Ar·Bi + Ai·Br          (4 DMMAs, 8 real flops / complex MAC)
 // with −Ai formed by flipping the sign bit (integer ALU, not the FP64 pipe).  No conjugation
 // anywhere (SURVEY.md §8(c) reading #7).
+#include <algorithm>
 #include <cstdio>
 #include <cstdlib>
 
@@ -1032,7 +1033,65 @@ __global__ void __launch_bounds__(DT) zdot_warp_kernel(const __grid_constant__ D
   zdot_warp_body(b.d, b.n, items);
 }
 
+// FP64 tensor-pipe ceiling probe: register-only DMMA chains (8 independent accumulators per
+// warp hide the DMMA latency), no memory traffic.  512 flops per DMMA.8x8x4.
+__global__ void __launch_bounds__(128) dmma_probe_kernel(double *out, int iters) {
+  double a = threadIdx.x * 1e-3, b = 1.0 + threadIdx.x * 1e-4;
+  double c[8][2];
+#pragma unroll
+  for (int i = 0; i < 8; ++i) c[i][0] = c[i][1] = 0.0;
+  for (int it = 0; it < iters; ++it) {
+#pragma unroll
+    for (int i = 0; i < 8; ++i) dmma(c[i][0], c[i][1], a, b);
+  }
+  double s = 0;
+#pragma unroll
+  for (int i = 0; i < 8; ++i) s += c[i][0] + c[i][1];
+  if (s == 12345.678) out[0] = s;  // (never true: keeps the chains live)
+}
+
 }  // namespace
+
+cudaError_t probe_fp64_peak(double seconds, double *burst_tflops, double *sustained_tflops) {
+  int dev = 0, sms = 148;
+  cudaError_t e;
+  if ((e = cudaGetDevice(&dev)) != cudaSuccess) return e;
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  double *out = nullptr;
+  if ((e = cudaMalloc(&out, 8)) != cudaSuccess) return e;
+  cudaStream_t st;
+  cudaStreamCreateWithFlags(&st, cudaStreamNonBlocking);
+  cudaEvent_t e0, e1;
+  cudaEventCreate(&e0);
+  cudaEventCreate(&e1);
+  const int iters = 4096, ctas = sms * 4;  // 4 CTAs × 4 warps = 16 warps per SM
+  const double flops = 512.0 * 8 * iters * (double)ctas * 4;
+  float best = 1e30f;
+  for (int rep = 0; rep < 5; ++rep) {  // burst: the best of a few single launches
+    cudaEventRecord(e0, st);
+    dmma_probe_kernel<<<ctas, 128, 0, st>>>(out, iters);
+    cudaEventRecord(e1, st);
+    cudaEventSynchronize(e1);
+    float ms = 0;
+    cudaEventElapsedTime(&ms, e0, e1);
+    if (ms > 0 && ms < best) best = ms;
+  }
+  *burst_tflops = flops / (best * 1e-3) * 1e-12;
+  const int n = std::max(1, (int)(seconds / (best * 1e-3)));
+  cudaEventRecord(e0, st);
+  for (int i = 0; i < n; ++i) dmma_probe_kernel<<<ctas, 128, 0, st>>>(out, iters);
+  cudaEventRecord(e1, st);
+  cudaEventSynchronize(e1);
+  float ms = 0;
+  cudaEventElapsedTime(&ms, e0, e1);
+  *sustained_tflops = flops * n / (ms * 1e-3) * 1e-12;
+  e = cudaGetLastError();
+  cudaEventDestroy(e0);
+  cudaEventDestroy(e1);
+  cudaStreamDestroy(st);
+  cudaFree(out);
+  return e;
+}
 
 int gemm_variant() {
   // MICCO_GEMM = 5 (default) persistent 64×32 tiles, 3M "T" complex products;

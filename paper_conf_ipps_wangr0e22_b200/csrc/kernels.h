@@ -99,4 +99,7 @@ cudaError_t launch_correlator_sum(int G, int Lt, const double2 *coefs, const dou
 // dst[i] += src[i] (exact: each slot is nonzero on exactly one source)
 cudaError_t launch_accumulate(double2 *dst, const double2 *src, long long n, cudaStream_t st);
 
+// FP64 DMMA ceiling of the current device (micco_probe_fp64_peak)
+cudaError_t probe_fp64_peak(double seconds, double *burst_tflops, double *sustained_tflops);
+
 }  // namespace micco

@@ -36,7 +36,7 @@ class micco_options(ctypes.Structure):
                 ("policy", ctypes.c_int32), ("window_graphs", ctypes.c_int32), ("seed", ctypes.c_uint64),
                 ("deterministic", ctypes.c_int32), ("keep_inputs_resident", ctypes.c_int32),
                 ("dist_rank", ctypes.c_int32), ("dist_world", ctypes.c_int32), ("reorder", ctypes.c_int32),
-                ("bound_model", ctypes.c_int32)]
+                ("bound_model", ctypes.c_int32), ("scalar_tables", ctypes.c_int32)]
 
 
 class micco_edge(ctypes.Structure):
@@ -56,7 +56,9 @@ class micco_stats(ctypes.Structure):
                 ("gemm_launches", ctypes.c_int64), ("dot_launches", ctypes.c_int64),
                 ("gemm_flops", ctypes.c_double), ("dot_bytes", ctypes.c_double),
                 ("enqueue_ms", ctypes.c_double), ("host_pinned", ctypes.c_int32), ("gemm_3m", ctypes.c_int32),
-                ("gemm_dmma_flops", ctypes.c_double)]
+                ("gemm_dmma_flops", ctypes.c_double), ("dot_main_ms", ctypes.c_double),
+                ("dot_main_bytes", ctypes.c_double), ("dot_main_launches", ctypes.c_int64),
+                ("plan_ms", ctypes.c_double)]
 
     def as_dict(self) -> Dict:
         d = {}
@@ -70,7 +72,8 @@ EXPORTS = ["micco_options_default", "micco_create", "micco_destroy", "micco_add_
            "micco_add_hadron_nodes_synth", "micco_add_graph", "micco_execute", "micco_get_correlator",
            "micco_get_graph_value", "micco_last_error", "micco_get_stats", "micco_release_cache",
            "micco_nccl_unique_id", "micco_set_nccl_id", "micco_plan", "micco_plan_ops", "micco_dag",
-           "micco_debug_schedule", "micco_plan_stages", "micco_predict_bounds"]
+           "micco_debug_schedule", "micco_plan_stages", "micco_predict_bounds", "micco_probe_fp64_peak",
+           "micco_set_policy"]
 
 _lib = None
 
@@ -117,7 +120,10 @@ def lib() -> ctypes.CDLL:
                                         P(ctypes.c_double), P(ctypes.c_int32), P(ctypes.c_int64), P(ctypes.c_double)]
         L.micco_predict_bounds.argtypes = [P(ctypes.c_double), P(ctypes.c_double), P(ctypes.c_int32)]
         L.micco_predict_bounds.restype = None
-        for f in ("micco_plan_stages", "micco_create", "micco_add_hadron_node", "micco_add_hadron_nodes_synth", "micco_add_graph",
+        L.micco_probe_fp64_peak.argtypes = [ctypes.c_double, P(ctypes.c_double), P(ctypes.c_double)]
+        L.micco_probe_fp64_peak.restype = ctypes.c_int
+        L.micco_set_policy.argtypes = [vp, ctypes.c_int32]
+        for f in ("micco_set_policy", "micco_plan_stages", "micco_create", "micco_add_hadron_node", "micco_add_hadron_nodes_synth", "micco_add_graph",
                   "micco_execute", "micco_get_correlator", "micco_get_graph_value", "micco_get_stats",
                   "micco_release_cache", "micco_nccl_unique_id", "micco_set_nccl_id", "micco_plan",
                   "micco_plan_ops", "micco_dag", "micco_debug_schedule"):
@@ -142,7 +148,7 @@ def _check(ctx, st: int):
 def micco_create(mem_budget_bytes: int = 0, policy: str = "micco", window_graphs: int = 0,
                  keep_inputs_resident: bool = False, dist_rank: int = 0, dist_world: int = 0,
                  deterministic: bool = True, seed: int = 0, reorder: bool = False,
-                 bound_model: int = 0) -> ctypes.c_void_p:
+                 bound_model: int = 0, scalar_tables: int = 0) -> ctypes.c_void_p:
     o = micco_options()
     lib().micco_options_default(ctypes.byref(o))
     o.mem_budget_bytes = int(mem_budget_bytes)
@@ -155,6 +161,7 @@ def micco_create(mem_budget_bytes: int = 0, policy: str = "micco", window_graphs
     o.seed = int(seed)
     o.reorder = 1 if reorder else 0
     o.bound_model = int(bound_model)
+    o.scalar_tables = int(scalar_tables)
     h = ctypes.c_void_p()
     _check(None, lib().micco_create(ctypes.byref(h), ctypes.byref(o)))
     return h
@@ -232,6 +239,10 @@ def micco_release_cache(ctx) -> None:
     _check(ctx, lib().micco_release_cache(ctx))
 
 
+def micco_set_policy(ctx, policy) -> None:
+    _check(ctx, lib().micco_set_policy(ctx, POLICIES[policy] if isinstance(policy, str) else int(policy)))
+
+
 def micco_plan(ctx, n_gpus: int, reuse_bound: Optional[Sequence[int]] = None, n_tasks: Optional[int] = None):
     s = micco_stats()
     s.struct_size = ctypes.sizeof(micco_stats)
@@ -283,6 +294,15 @@ def micco_predict_bounds(features: Sequence[float]):
     b = np.zeros(3, dtype=np.int32)
     lib().micco_predict_bounds(_ptr(f, ctypes.c_double), _ptr(raw, ctypes.c_double), _ptr(b, ctypes.c_int32))
     return raw, b
+
+
+def micco_probe_fp64_peak(seconds: float = 1.0):
+    """(burst, sustained) FP64 DMMA TFLOP/s of the current device (register-only loop)."""
+    b, s = ctypes.c_double(), ctypes.c_double()
+    st = lib().micco_probe_fp64_peak(float(seconds), ctypes.byref(b), ctypes.byref(s))
+    if st != MICCO_OK:
+        raise MiccoError(st, "probe_fp64_peak")
+    return b.value, s.value
 
 
 def micco_dag(ctx):
@@ -392,6 +412,9 @@ class Context:
 
     def release_cache(self):
         micco_release_cache(self.h)
+
+    def set_policy(self, policy):
+        micco_set_policy(self.h, policy)
 
 
 def load_workload(ctx: Context, wl, node_arrays: Optional[Sequence[np.ndarray]] = None) -> List[int]:
