@@ -223,6 +223,8 @@ typedef struct {
   int64_t dot_main_launches;
   double plan_ms;              /* host time of make_plan for this execute (overlapped with the
                                   replay when planning streams; sched_ms = the same) */
+  int64_t gemm_tma_launches;   /* GEMM launches on the TMA warp-specialized kernel (the rest ran on
+                                  the cp.async kernels: ragged k, odd rows, 6-D views) */
 } micco_stats;
 
 MICCO_API micco_status micco_get_stats(const micco_ctx *ctx, micco_stats *out);

@@ -19,6 +19,7 @@
 #include <nccl.h>
 
 #include <algorithm>
+#include <array>
 #include <chrono>
 #include <cstdlib>
 #include <cstring>
@@ -160,6 +161,7 @@ struct LGpu {
   std::vector<double2 *> ptr;                                  // tensor → replica
   std::unordered_map<int32_t, std::vector<cudaEvent_t>> readers;  // peer reads to wait for before free
   std::vector<GemmDesc> gemm;
+  std::vector<std::array<CUtensorMap, 2>> gemm_maps;  // per gemm entry (TMA classes only)
   std::vector<DotDesc> dot;
   std::vector<double2 *> part_allocs;  // fused-dot partials of the pending batch
   long long gemm_tiles = 0, dot_ctas = 0;
@@ -188,6 +190,7 @@ struct Executor::Impl {
   std::vector<std::pair<int32_t, uint64_t>> cached_nodes;
   std::vector<int32_t> fused_dot;  // of the plan being replayed
   std::unique_ptr<GemmBatch> gemm_batch{new GemmBatch};  // kernel-parameter staging
+  std::unique_ptr<GemmTmaBatch> tma_batch{new GemmTmaBatch};
   std::unique_ptr<DotBatch> dot_batch{new DotBatch};
   int32_t chosen_bd[3] = {0, 0, 0};
   int chosen_bd_n = 0;
@@ -200,7 +203,7 @@ struct Executor::Impl {
   size_t vals_elems = 0;
   int vals_dev = 0;
   double2 *h_corr = nullptr;
-  int64_t launches = 0;
+  int64_t launches = 0, tma_launches = 0;
   bool dist() const { return c.opt.dist_world > 0; }
   int table_of(int i) const { return c.opt.scalar_tables ? i : g[i].dev; }
   double2 *table_row(const LGpu &l, int32_t slot) const {
@@ -460,9 +463,38 @@ struct Executor::Impl {
     CK(cudaSetDevice(l.dev));
     if (!l.gemm.empty()) {  // one grouped launch per operand-layout class
       std::vector<GemmDesc> by[kGemmClasses];
-      for (const GemmDesc &d : l.gemm) by[d.cls].push_back(d);
+      std::vector<size_t> tma_idx[kGemmClasses];
+      for (size_t i = 0; i < l.gemm.size(); ++i) {
+        const GemmDesc &d = l.gemm[i];
+        if (d.cls >= kGemmClassTMA) tma_idx[d.cls].push_back(i);
+        else by[d.cls].push_back(d);
+      }
+      for (int c = kGemmClassTMA; c < kGemmClasses; ++c) {  // TMA kernel: descriptors + tensor maps
+        const std::vector<size_t> &ix = tma_idx[c];
+        for (size_t i0 = 0; i0 < ix.size(); i0 += kGemmTmaBatch) {
+          const int cnt = (int)std::min((size_t)kGemmTmaBatch, ix.size() - i0);
+          GemmTmaBatch &b = *tma_batch;
+          b.n = cnt;
+          long long acc = 0;
+          for (int k = 0; k < cnt; ++k) {
+            b.d[k] = l.gemm[ix[i0 + k]];
+            b.map[2 * k] = l.gemm_maps[ix[i0 + k]][0];
+            b.map[2 * k + 1] = l.gemm_maps[ix[i0 + k]][1];
+            b.d[k].tile_begin = acc;
+            acc += (long long)b.d[k].Lt * b.d[k].Mo * b.d[k].No * b.d[k].tilesM * b.d[k].tilesN;
+          }
+          Timed tm{devs[l.dev].timing_events.get(), devs[l.dev].timing_events.get(), 0, l.dev};
+          CK(cudaEventRecord(tm.a, l.st));
+          CK(launch_gemm_tma_group(&b, acc, c, l.st));
+          CK(cudaEventRecord(tm.b, l.st));
+          timed.push_back(tm);
+          ++launches;
+          ++tma_launches;
+        }
+      }
       l.gemm.clear();
-      for (int c = 0; c < kGemmClasses; ++c)
+      l.gemm_maps.clear();
+      for (int c = 0; c < kGemmClassTMA; ++c)
         launch_batch(l, by[c], 0, c, *gemm_batch, kGemmBatch, [](GemmDesc *d, int cnt) {
           long long acc = 0;
           for (int i = 0; i < cnt; ++i) {
@@ -518,6 +550,11 @@ struct Executor::Impl {
       d.sCmo = L.sCmo; d.sCmi = L.sCmi; d.sCno = L.sCno; d.sCni = L.sCni;
       d.Lt = c.Lt;
       d.cls = gemm_kernel_class(gemm_class(L), L.Ko);
+      std::array<CUtensorMap, 2> maps;
+      {
+        int tcls;  // the TMA kernel when the operands fit its tensor maps (kernels.cu gemm_tma_class)
+        if (gemm_tma_class(d, &tcls) && gemm_tma_encode(d, tcls, &maps[0], &maps[1])) d.cls = tcls;
+      }
       int tbm, tbn;
       gemm_tile_shape(d.cls, &tbm, &tbn);
       d.tilesM = (L.Mi + tbm - 1) / tbm;
@@ -539,7 +576,7 @@ struct Executor::Impl {
         d.sDmo = d.sDno = 0;
         d.sDmi = sY[q[0]];
         d.sDni = sY[q[1]];
-        const long long tps = (long long)L.Mo * L.No * d.tilesM * d.tilesN * 4;  // partials per slice
+        const long long tps = (long long)L.Mo * L.No * d.tilesM * d.tilesN * gemm_warps_per_tile(d.cls);  // partials per slice
         d.part = alloc(l, tps * c.Lt * 16);
         l.part_allocs.push_back(d.part);
         DotDesc r{};
@@ -551,6 +588,7 @@ struct Executor::Impl {
         st.dot_bytes += (double)YT.slice_elems * 16.0 * c.Lt;
       }
       l.gemm.push_back(d);
+      l.gemm_maps.push_back(maps);
       st.gemm_flops += tk.flops;
       const bool m3 = gemm_uses_3m(d.cls);
       st.gemm_dmma_flops += m3 ? tk.flops * 0.75 : tk.flops;
@@ -746,6 +784,7 @@ struct Executor::Impl {
       for (double2 *p : l.part_allocs) cudaFree(p);
       l.part_allocs.clear();
       l.gemm.clear();
+      l.gemm_maps.clear();
       l.dot.clear();
       l.readers.clear();
       l.flush_ev.clear();
@@ -767,6 +806,7 @@ struct Executor::Impl {
     for (auto &l : g)
       if (l.local && l.ptr.size() < c.tensors.size()) l.ptr.resize(c.tensors.size(), nullptr);
     launches = 0;
+    tma_launches = 0;
     timed.clear();
     for (auto &l : g) {
       l.flush_ev.clear();
@@ -1050,6 +1090,7 @@ struct Executor::Impl {
     for (const TaskRec &t : c.tasks) (t.kind == TASK_GEMM ? st.n_gemm : st.n_dot)++;
     st.n_stages = plan.n_stages;
     st.kernel_launches = launches;
+    st.gemm_tma_launches = tma_launches;
     st.flops = plan.flops;
     for (const GraphRec &gr : c.graphs) st.flops_no_dedup += gr.flops_no_dedup;
     st.max_over_mean_load = plan.max_over_mean_load;

@@ -15,6 +15,8 @@
 #include <cstdio>
 #include <cstdlib>
 
+#include <cudaTypedefs.h>
+
 #include "kernels.h"
 
 namespace micco {
@@ -749,6 +751,314 @@ __device__ __forceinline__ void zgemm_persistent_body(const GemmDesc *__restrict
   cp_async_wait<0>();
 }
 
+// ---------------------------------------------------------------- TMA warp-specialized GEMM (3M)
+//
+// The production GEMM for contractions whose operands fit 5-D tensor maps (every meson GEMM;
+// gemm_tma_class).  One CTA per SM: two consumer warpgroups (8 warps, 4 × 2, warp tile 32 × 16
+// complex, 3M "T" accumulators; CTA tile 128 × 32) and one producer warpgroup whose elected lane
+// streams the operand stages with TMA (cp.async.bulk.tensor, SASS UTMALDG) through a 5-slot
+// shared-memory ring guarded by full/empty mbarriers.  Registers are allocated per warpgroup
+// (a 9-warp CTA is charged for 12): the kernel launches at 168 per thread, then the producer
+// warpgroup gives back to 40 and the consumers grow to 232 (setmaxnreg).  The consumers' loop is fragment LDS + operand-sum DADD + DMMA plus one
+// mbarrier wait and one arrive per stage: no per-thread copy addressing, no bounds masks (TMA
+// zero-fills ragged tiles) and no CTA-wide barrier (the cp.async kernel above spent ~180
+// non-DMMA instructions per 96 DMMAs per stage on them, ncu profiles/ncu_gemm_c3_r02.json).
+//
+// The tensor maps lay each stage out for conflict-free 16-byte fragment loads without padding
+// (probe: tools/tma_probe.cu):
+//   K-major operand (contiguous along k):   smem [kq][row][k4]      (lane (r, c) of an 8-row
+//                                           block reads 32 consecutive complex)
+//   MN-major operand (contiguous along row): smem [kq][row/2][k4][2] (lanes 0-7 = rows 0-1 ×
+//                                           k 0-3 hit 8 distinct 16-byte bank groups)
+// where kq = k / 4 and k4 = k % 4: the map's dimensions step through the operand in that order
+// (non-monotonic global strides, accepted by cuTensorMapEncodeTiled).
+constexpr int TM_NWM = 4, TM_NWN = 2, TM_NW = TM_NWM * TM_NWN;  // consumer warps
+constexpr int TM_BM = TM_NWM * 32, TM_BN = TM_NWN * 16, TM_BK = 16, TM_ST = 5;
+constexpr int TM_THREADS = (TM_NW + 4) * 32;  // + the producer warpgroup
+constexpr int TM_REG_LAUNCH = 168, TM_REG_PRODUCER = 40, TM_REG_CONSUMER = 232;
+static_assert(TM_THREADS * TM_REG_LAUNCH <= 65536, "register file");
+static_assert(4 * 32 * (TM_REG_LAUNCH - TM_REG_PRODUCER) >= TM_NW * 32 * (TM_REG_CONSUMER - TM_REG_LAUNCH),
+              "setmaxnreg balance");
+constexpr int TM_AE = TM_BM * TM_BK, TM_BE = TM_BN * TM_BK;  // complex per stage
+constexpr int TM_STAGE_BYTES = (TM_AE + TM_BE) * 16;
+constexpr int TM_SMEM = TM_ST * TM_STAGE_BYTES + 2 * TM_ST * 8;
+
+__device__ __forceinline__ unsigned smem_u32(const void *p) { return (unsigned)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mbar_init(unsigned bar, unsigned cnt) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(bar), "r"(cnt) : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(unsigned bar, unsigned bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(unsigned bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(bar) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(unsigned bar, unsigned parity) {
+  asm volatile(
+      "{\n .reg .pred p;\n TMW_%=: mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n @!p bra TMW_%=;\n}\n" ::"r"(bar),
+      "r"(parity)
+      : "memory");
+}
+__device__ __forceinline__ void tma_load5(unsigned dst, const CUtensorMap *m, unsigned bar, int c0, int c1, int c2, int c3,
+                                          int c4) {
+  asm volatile(
+      "cp.async.bulk.tensor.5d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4, %5, %6}], [%7];" ::"r"(
+          dst),
+      "l"(m), "r"(c0), "r"(c1), "r"(c2), "r"(c3), "r"(c4), "r"(bar)
+      : "memory");
+}
+
+// tile → (task, t, mo, no, m0, n0); descriptors advance linearly (tiles increase)
+struct TmTile {
+  int t, mo, no, m0, n0;
+};
+__device__ __forceinline__ TmTile tm_decode(const GemmDesc *__restrict__ descs, int n_desc, int &task, long long tile) {
+  while (task + 1 < n_desc && descs[task + 1].tile_begin <= tile) ++task;
+  const GemmDesc &d = descs[task];
+  unsigned lt = (unsigned)(tile - d.tile_begin);  // < 2^32 tiles per task (executor.cu check)
+  TmTile r;
+  const unsigned tilesN = d.tilesN, tilesM = d.tilesM, No = d.No, Mo = d.Mo;
+  const int tn = (int)(lt % tilesN); lt /= tilesN;
+  const int tm = (int)(lt % tilesM); lt /= tilesM;
+  r.no = (int)(lt % No); lt /= No;
+  r.mo = (int)(lt % Mo);
+  r.t = (int)(lt / Mo);
+  r.m0 = tm * TM_BM;
+  r.n0 = tn * TM_BN;
+  return r;
+}
+
+// Fragment offset (complex) of lane within an 8-row block, per operand layout.
+template <bool KMAJ>
+__device__ __forceinline__ int tm_lane_off(int lane) {
+  if constexpr (KMAJ) return lane;                        // row·4 + k4
+  const int r = lane >> 2, c = lane & 3;
+  return (r >> 1) * 8 + c * 2 + (r & 1);                 // (row/2)·8 + k4·2 + row%2
+}
+
+template <bool AK, bool BK>
+__device__ __forceinline__ void zgemm_tma_body(const GemmTmaBatch &b, long long total) {
+  constexpr int MI = 4, NJ = 2;  // 8×8 blocks per warp (32 × 16 complex)
+  extern __shared__ __align__(128) double2 smem[];
+  double2 *As = smem;                    // [TM_ST][TM_AE]
+  double2 *Bs = smem + TM_ST * TM_AE;    // [TM_ST][TM_BE]
+  unsigned long long *bars = reinterpret_cast<unsigned long long *>(Bs + TM_ST * TM_BE);
+  const unsigned full0 = smem_u32(bars), empty0 = smem_u32(bars + TM_ST);
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const GemmDesc *__restrict__ descs = b.d;
+  const int n_desc = b.n;
+  const long long G = gridDim.x;
+  if (tid == 0) {
+    for (int i = 0; i < TM_ST; ++i) {
+      mbar_init(full0 + 8 * i, 1);   // the producer's arrive.expect_tx (+ the TMA bytes)
+      mbar_init(empty0 + 8 * i, TM_NW);  // one arrive per consumer warp
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+  if ((long long)blockIdx.x >= total) return;
+  int task0 = 0;
+  {
+    int lo = 0, hi = n_desc - 1;
+    while (lo < hi) {
+      const int mid = (lo + hi + 1) >> 1;
+      if (descs[mid].tile_begin <= (long long)blockIdx.x) lo = mid; else hi = mid - 1;
+    }
+    task0 = lo;
+  }
+
+  if (warp >= TM_NW) {  // ---------------- producer warpgroup: one lane streams every stage
+    asm volatile("setmaxnreg.dec.sync.aligned.u32 %0;" ::"n"(TM_REG_PRODUCER));
+    if (warp != TM_NW || lane != 0) return;
+    int task = task0, slot = 0;
+    unsigned ph = 0;
+    int prefetched = -1;
+    for (long long tile = blockIdx.x; tile < total; tile += G) {
+      const TmTile tt = tm_decode(descs, n_desc, task, tile);
+      const GemmDesc &d = descs[task];
+      const CUtensorMap *ma = &b.map[2 * task], *mb = &b.map[2 * task + 1];
+      if (task != prefetched) {
+        asm volatile("prefetch.tensormap [%0];" ::"l"(ma) : "memory");
+        asm volatile("prefetch.tensormap [%0];" ::"l"(mb) : "memory");
+        prefetched = task;
+      }
+      const int kti = (d.Ki + TM_BK - 1) / TM_BK;
+      const int ks_n = d.Ko * kti;
+      for (int ks = 0; ks < ks_n; ++ks) {
+        const int ko = ks / kti, kq0 = (ks - ko * kti) * (TM_BK / 4);
+        mbar_wait(empty0 + 8 * slot, ph ^ 1);
+        const unsigned fb = full0 + 8 * slot;
+        mbar_expect_tx(fb, TM_STAGE_BYTES);
+        const unsigned sa = smem_u32(As + slot * TM_AE), sb = smem_u32(Bs + slot * TM_BE);
+        if constexpr (AK) tma_load5(sa, ma, fb, 0, tt.m0, kq0, tt.t, d.Ko > 1 ? ko : tt.mo);
+        else tma_load5(sa, ma, fb, 0, 0, tt.m0 >> 1, kq0, tt.t);
+        if constexpr (BK) tma_load5(sb, mb, fb, 0, tt.n0, kq0, tt.t, d.Ko > 1 ? ko : tt.no);
+        else tma_load5(sb, mb, fb, 0, 0, tt.n0 >> 1, kq0, tt.t);
+        if (++slot == TM_ST) { slot = 0; ph ^= 1; }
+      }
+    }
+    return;
+  }
+
+  // ---------------- consumers: TM_NWM × TM_NWN warps
+  asm volatile("setmaxnreg.inc.sync.aligned.u32 %0;" ::"n"(TM_REG_CONSUMER));
+  const int wm = warp / TM_NWN, wn = warp % TM_NWN;
+  const int aoff = wm * 128 + tm_lane_off<AK>(lane);  // + kq·(TM_BM·4) + i·32
+  const int boff = wn * 64 + tm_lane_off<BK>(lane);   // + kq·(TM_BN·4) + j·32
+  double acc[MI][NJ][3][2];
+#pragma unroll
+  for (int i = 0; i < MI; ++i)
+#pragma unroll
+    for (int j = 0; j < NJ; ++j)
+#pragma unroll
+      for (int q = 0; q < 3; ++q) acc[i][j][q][0] = acc[i][j][q][1] = 0.0;
+  double fa[2][MI][3], fb[2][NJ][3];
+  auto load_frag = [&](int buf, int slot, int kq) {
+    const double2 *as = As + slot * TM_AE + kq * (TM_BM * 4) + aoff;
+    const double2 *bs = Bs + slot * TM_BE + kq * (TM_BN * 4) + boff;
+#pragma unroll
+    for (int i = 0; i < MI; ++i) {
+      const double2 a = as[i * 32];
+      fa[buf][i][0] = a.x;
+      fa[buf][i][1] = a.y;
+      fa[buf][i][2] = a.x + a.y;  // Ar + Ai
+    }
+#pragma unroll
+    for (int j = 0; j < NJ; ++j) {
+      const double2 v = bs[j * 32];
+      fb[buf][j][0] = v.x;
+      fb[buf][j][1] = v.y;
+      fb[buf][j][2] = v.x + v.y;  // Br + Bi
+    }
+  };
+
+  int task = task0, slot = 0;
+  unsigned ph = 0;
+  long long tile = blockIdx.x;
+  TmTile tt = tm_decode(descs, n_desc, task, tile);
+  int ks_n = descs[task].Ko * ((descs[task].Ki + TM_BK - 1) / TM_BK);
+  int ks = 0;
+  mbar_wait(full0, 0);
+  load_frag(0, 0, 0);
+  for (;;) {
+#pragma unroll
+    for (int kq = 0; kq < TM_BK / 4; ++kq) {
+      const int cur = kq & 1;
+      if (kq + 1 < TM_BK / 4) {
+        load_frag(cur ^ 1, slot, kq + 1);
+      } else {
+        // every fragment of this slot is in registers (and summed): hand the slot back
+        __syncwarp();
+        if (lane == 0) mbar_arrive(empty0 + 8 * slot);
+        if (++slot == TM_ST) { slot = 0; ph ^= 1; }
+        if (ks + 1 < ks_n) {  // (the next tile's first fragments are loaded after the epilogue)
+          mbar_wait(full0 + 8 * slot, ph);
+          load_frag(cur ^ 1, slot, 0);
+        }
+      }
+#pragma unroll
+      for (int i = 0; i < MI; ++i)
+#pragma unroll
+        for (int j = 0; j < NJ; ++j) {
+          dmma(acc[i][j][0][0], acc[i][j][0][1], fa[cur][i][0], fb[cur][j][0]);  // Ar·Br
+          dmma(acc[i][j][1][0], acc[i][j][1][1], fa[cur][i][1], fb[cur][j][1]);  // Ai·Bi
+          dmma(acc[i][j][2][0], acc[i][j][2][1], fa[cur][i][2], fb[cur][j][2]);  // (Ar+Ai)·(Br+Bi)
+        }
+    }
+    const GemmDesc &dd = descs[task];
+    if (dd.D && ks + 2 == ks_n) {
+      // fused dot: pull this tile's partner block into L2 one stage before the epilogue
+      const double2 *D = dd.D + tt.t * dd.sDt + tt.mo * dd.sDmo + tt.no * dd.sDno;
+      const bool mrow = dd.sDni == 1;
+      const int rows = mrow ? min(TM_BM, dd.Mi - tt.m0) : min(TM_BN, dd.Ni - tt.n0);
+      const int segs = (mrow ? TM_BN : TM_BM) / 8;
+      for (int q = tid; q < rows * segs; q += TM_NW * 32) {
+        const int r = q / segs, seg = (q % segs) * 8;
+        const double2 *pp = mrow ? D + (long long)(tt.m0 + r) * dd.sDmi + tt.n0 + seg
+                                 : D + (long long)(tt.n0 + r) * dd.sDni + tt.m0 + seg;
+        asm volatile("prefetch.global.L2 [%0];\n" ::"l"(pp));
+      }
+    }
+    if (++ks < ks_n) continue;
+    // ---- tile done: 3M combine, then store C or the fused dot's partial sum
+    {
+      const int Mi = dd.Mi, Ni = dd.Ni;
+      auto cval = [&](int i, int j, int h, double &re, double &im) {
+        re = acc[i][j][0][h] - acc[i][j][1][h];
+        im = acc[i][j][2][h] - (acc[i][j][0][h] + acc[i][j][1][h]);
+      };
+      if (dd.D) {
+        const double2 *D = dd.D + tt.t * dd.sDt + tt.mo * dd.sDmo + tt.no * dd.sDno;
+        const long long sDmi = dd.sDmi, sDni = dd.sDni;
+        double pr = 0.0, pim = 0.0;
+        constexpr int CH = MI;  // partner rows in flight
+#pragma unroll
+        for (int i0 = 0; i0 < MI; i0 += CH) {
+          double2 y[CH][NJ][2];
+#pragma unroll
+          for (int ii = 0; ii < CH; ++ii) {
+            const int m = tt.m0 + wm * 32 + (i0 + ii) * 8 + (lane >> 2);
+#pragma unroll
+            for (int j = 0; j < NJ; ++j)
+#pragma unroll
+              for (int h = 0; h < 2; ++h) {
+                const int n = tt.n0 + wn * 16 + j * 8 + (lane & 3) * 2 + h;
+                y[ii][j][h] = (m < Mi && n < Ni) ? D[(long long)m * sDmi + (long long)n * sDni] : make_double2(0.0, 0.0);
+              }
+          }
+#pragma unroll
+          for (int ii = 0; ii < CH; ++ii)
+#pragma unroll
+            for (int j = 0; j < NJ; ++j)
+#pragma unroll
+              for (int h = 0; h < 2; ++h) {
+                double re, im;
+                cval(i0 + ii, j, h, re, im);
+                pr += re * y[ii][j][h].x - im * y[ii][j][h].y;
+                pim += re * y[ii][j][h].y + im * y[ii][j][h].x;
+              }
+        }
+#pragma unroll
+        for (int off = 16; off > 0; off >>= 1) {
+          pr += __shfl_xor_sync(0xffffffffu, pr, off);
+          pim += __shfl_xor_sync(0xffffffffu, pim, off);
+        }
+        if (lane == 0) dd.part[(tile - dd.tile_begin) * TM_NW + warp] = make_double2(pr, pim);
+      } else {
+        double2 *C = dd.C + tt.t * dd.sCt + tt.mo * dd.sCmo + tt.no * dd.sCno;
+        const long long sCmi = dd.sCmi, sCni = dd.sCni;
+#pragma unroll
+        for (int i = 0; i < MI; ++i) {
+          const int m = tt.m0 + wm * 32 + i * 8 + (lane >> 2);
+          if (m >= Mi) continue;
+#pragma unroll
+          for (int j = 0; j < NJ; ++j) {
+            const int n = tt.n0 + wn * 16 + j * 8 + (lane & 3) * 2;
+            double2 *cp = C + (long long)m * sCmi + (long long)n * sCni;
+            double re, im;
+            cval(i, j, 0, re, im);
+            if (n < Ni) cp[0] = make_double2(re, im);
+            cval(i, j, 1, re, im);
+            if (n + 1 < Ni) cp[sCni] = make_double2(re, im);
+          }
+        }
+      }
+    }
+#pragma unroll
+    for (int i = 0; i < MI; ++i)
+#pragma unroll
+      for (int j = 0; j < NJ; ++j)
+#pragma unroll
+        for (int q = 0; q < 3; ++q) acc[i][j][q][0] = acc[i][j][q][1] = 0.0;
+    if ((tile += G) >= total) break;
+    tt = tm_decode(descs, n_desc, task, tile);
+    ks_n = descs[task].Ko * ((descs[task].Ki + TM_BK - 1) / TM_BK);
+    ks = 0;
+    mbar_wait(full0 + 8 * slot, ph);
+    load_frag(0, slot, 0);
+  }
+}
+
 // ---------------------------------------------------------------- dot / trace
 
 constexpr int DT = 256;
@@ -1028,6 +1338,11 @@ void (*persistent_fn(int cls))(const GemmBatch, long long, unsigned) {
   }
 }
 
+template <bool AK, bool BK>
+__global__ void __launch_bounds__(TM_THREADS, 1) zgemm_tma(const __grid_constant__ GemmTmaBatch b, long long total) {
+  zgemm_tma_body<AK, BK>(b, total);
+}
+
 __global__ void __launch_bounds__(DT, MICCO_DOT_MINB) zdot_kernel(const __grid_constant__ DotBatch b) { zdot_body(b.d, b.n); }
 __global__ void __launch_bounds__(DT) zdot_warp_kernel(const __grid_constant__ DotBatch b, long long items) {
   zdot_warp_body(b.d, b.n, items);
@@ -1111,11 +1426,14 @@ int gemm_variant() {
 void gemm_tile_shape(int cls, int *bm, int *bn) {
   *bm = 64;
   *bn = 64;
+  if (cls >= kGemmClassTMA) { *bm = TM_BM; *bn = TM_BN; return; }
   if (cls == 4) return;  // gather kernel (v1)
   if (gemm_variant() >= 5) *bn = 32;
 }
 
 bool gemm_uses_3m(int cls) { return cls != 4 && gemm_variant() >= 5; }
+
+int gemm_warps_per_tile(int cls) { return cls >= kGemmClassTMA ? TM_NW : 4; }
 
 int gemm_kernel_class(int layout_cls, int Ko) {
   // class 4 (no unit stride on an operand's free or inner contracted index) goes to the
@@ -1194,6 +1512,99 @@ cudaError_t launch_gemm_group(const GemmBatch *b, long long total_tiles, int cls
   else  // 6: the 3M "K" form
     persistent_fn<2, 2, 32, 16, true, false>(cls)<<<(unsigned)grid, 128, PCfg<64, 32>::SMEM, st>>>(*b, total_tiles,
                                                                                           (unsigned)phase_ns);
+  return cudaGetLastError();
+}
+
+bool gemm_tma_class(const GemmDesc &d, int *cls) {
+  static int off = -1;  // MICCO_GEMM_TMA=0: keep every contraction on the cp.async kernels
+  if (off < 0) {
+    const char *e = getenv("MICCO_GEMM_TMA");
+    off = (e && e[0] == '0') ? 1 : 0;
+  }
+  if (off || gemm_variant() != 5) return false;
+  const bool ak = d.sAki == 1, bk = d.sBki == 1;  // K-major operands (else contiguous along m / n)
+  if (!ak && d.sAmi != 1) return false;
+  if (!bk && d.sBni != 1) return false;
+  if (d.Ki % 4 != 0) return false;  // k-quads are the maps' inner unit
+  // 5 dimensions per map: K-major (k4, row, kq, t, outer-or-ko), MN-major (row pair, k4, row/2, kq, t)
+  if (ak ? (d.Ko > 1 && d.Mo > 1) : (d.Ko > 1 || d.Mo > 1 || d.Mi % 2 != 0)) return false;
+  if (bk ? (d.Ko > 1 && d.No > 1) : (d.Ko > 1 || d.No > 1 || d.Ni % 2 != 0)) return false;
+  if ((((uintptr_t)d.A) | ((uintptr_t)d.B)) & 15) return false;
+  *cls = kGemmClassTMA + (ak ? 0 : 2) + (bk ? 1 : 0);
+  return true;
+}
+
+namespace {
+PFN_cuTensorMapEncodeTiled_v12000 tensor_map_encoder() {
+  static PFN_cuTensorMapEncodeTiled_v12000 fn = [] {
+    void *f = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &f, cudaEnableDefault, &q) != cudaSuccess ||
+        q != cudaDriverEntryPointSuccess)
+      f = nullptr;
+    return (PFN_cuTensorMapEncodeTiled_v12000)f;
+  }();
+  return fn;
+}
+
+// One operand's map.  rows/srow: its free index inside the tile (m or n) and stride; sk: the
+// inner contracted stride; Ki; Lt and the slice stride; outer: (size, stride) of the 5th
+// K-major dimension (Ko when > 1, else the operand's outer free index).  Strides in complex.
+bool encode_operand(CUtensorMap *m, const double2 *base, bool kmaj, int rows, long long srow, long long sk, int Ki,
+                    int Lt, long long st, int box_rows, long long outer_n, long long outer_s) {
+  auto enc = tensor_map_encoder();
+  if (!enc) return false;
+  cuuint64_t dims[5], str[4];
+  cuuint32_t box[5], es[5] = {1, 1, 1, 1, 1};
+  if (kmaj) {  // (k4 as 8 doubles, row, kq, t, outer) → smem [kq][row][k4]
+    dims[0] = 8; dims[1] = rows; dims[2] = Ki / 4; dims[3] = Lt; dims[4] = outer_n;
+    str[0] = srow * 16; str[1] = 64; str[2] = st * 16; str[3] = (outer_n > 1 ? outer_s : 1) * 16;
+    box[0] = 8; box[1] = box_rows; box[2] = TM_BK / 4; box[3] = 1; box[4] = 1;
+  } else {     // (row pair as 4 doubles, k4, row/2, kq, t) → smem [kq][row/2][k4][2]
+    dims[0] = 4; dims[1] = 4; dims[2] = rows / 2; dims[3] = Ki / 4; dims[4] = Lt;
+    str[0] = sk * 16; str[1] = 32; str[2] = sk * 4 * 16; str[3] = st * 16;
+    box[0] = 4; box[1] = 4; box[2] = box_rows / 2; box[3] = TM_BK / 4; box[4] = 1;
+  }
+  for (int i = 0; i < 4; ++i)
+    if (str[i] == 0 || str[i] % 16 != 0 || str[i] >= (1ull << 40)) return false;
+  return enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 5, (void *)base, dims, str, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+             CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
+             CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
+}  // namespace
+
+bool gemm_tma_encode(const GemmDesc &d, int cls, CUtensorMap *a, CUtensorMap *b) {
+  const int c = cls - kGemmClassTMA;
+  const bool ak = (c & 2) == 0, bk = (c & 1) != 0;
+  const long long aon = d.Ko > 1 ? d.Ko : d.Mo, aos = d.Ko > 1 ? d.sAko : d.sAmo;
+  const long long bon = d.Ko > 1 ? d.Ko : d.No, bos = d.Ko > 1 ? d.sBko : d.sBno;
+  return encode_operand(a, d.A, ak, d.Mi, ak ? d.sAmi : 1, ak ? 1 : d.sAki, d.Ki, d.Lt, d.sAt, TM_BM, aon, aos) &&
+         encode_operand(b, d.B, bk, d.Ni, bk ? d.sBni : 1, bk ? 1 : d.sBki, d.Ki, d.Lt, d.sBt, TM_BN, bon, bos);
+}
+
+cudaError_t launch_gemm_tma_group(const GemmTmaBatch *b, long long total_tiles, int cls, cudaStream_t st) {
+  static unsigned long long attr_set = 0;  // per device (see launch_gemm_group)
+  int dev = 0;
+  if (cudaError_t e = cudaGetDevice(&dev); e != cudaSuccess) return e;
+  const unsigned long long bit = 1ull << (dev & 63);
+  if (!(attr_set & bit)) {
+    for (auto fn : {zgemm_tma<true, true>, zgemm_tma<true, false>, zgemm_tma<false, true>, zgemm_tma<false, false>}) {
+      cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, TM_SMEM);
+      if (e != cudaSuccess) return e;
+    }
+    attr_set |= bit;
+  }
+  if (total_tiles <= 0) return cudaSuccess;
+  int sms = 148;
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  long long grid = sms;  // one resident CTA per SM (TM_NW consumer warps + the producer)
+  if (grid > total_tiles) grid = total_tiles;
+  switch (cls - kGemmClassTMA) {
+    case 0: zgemm_tma<true, false><<<(unsigned)grid, TM_THREADS, TM_SMEM, st>>>(*b, total_tiles); break;
+    case 1: zgemm_tma<true, true><<<(unsigned)grid, TM_THREADS, TM_SMEM, st>>>(*b, total_tiles); break;
+    case 2: zgemm_tma<false, false><<<(unsigned)grid, TM_THREADS, TM_SMEM, st>>>(*b, total_tiles); break;
+    default: zgemm_tma<false, true><<<(unsigned)grid, TM_THREADS, TM_SMEM, st>>>(*b, total_tiles); break;
+  }
   return cudaGetLastError();
 }
 

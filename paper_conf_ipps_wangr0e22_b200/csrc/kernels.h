@@ -4,6 +4,7 @@
 #pragma once
 
 #include <cstdint>
+#include <cuda.h>  // CUtensorMap (the type only: tensor maps are encoded through the runtime's driver entry point)
 #include <cuda_runtime.h>
 
 namespace micco {
@@ -73,18 +74,40 @@ static_assert(sizeof(GemmBatch) <= 32764 && sizeof(DotBatch) <= 32764, "kernel p
 // GEMM descriptors carry their operand-layout class (layout.h gemm_class): 0..3 = unit-stride
 // inner index for both operands (warp-specialized kernel), 4 = generic gather kernel.
 // 5 = class 4 on the blocked-K persistent kernel (gemm_kernel_class).
-constexpr int kGemmClassKB = 5, kGemmClasses = 6;
+constexpr int kGemmClassKB = 5;
+// 6..9 = the TMA warp-specialized kernel, kGemmClassTMA + (A contiguous along m ? 2 : 0) +
+// (B contiguous along k ? 1 : 0), for contractions whose operands fit its tensor maps
+// (gemm_tma_class); everything else stays on classes 0..5.
+constexpr int kGemmClassTMA = 6, kGemmClasses = 10;
+
+// A grouped launch of the TMA kernel: two tensor maps per descriptor (A, B), 64-byte aligned
+// inside the __grid_constant__ parameter, then the descriptors.
+constexpr int kGemmTmaBatch = 48;
+struct GemmTmaBatch {
+  CUtensorMap map[2 * kGemmTmaBatch];
+  int n, pad[15];
+  GemmDesc d[kGemmTmaBatch];
+};
+static_assert(sizeof(GemmTmaBatch) <= 32764, "kernel parameter limit");
+
+// The TMA class of a descriptor (its strides and extents set, tile counts not yet), or false
+// when its operands do not fit the kernel's 5-D tensor maps (then it keeps its class).
+bool gemm_tma_class(const GemmDesc &d, int *cls);
+// Encode the two operand tensor maps of a TMA-class descriptor (host; no device work).
+bool gemm_tma_encode(const GemmDesc &d, int cls, CUtensorMap *a, CUtensorMap *b);
 
 // The GEMM kernel variant in use (env MICCO_GEMM, see kernels.cu) and its CTA tile (complex
 // elements) for a layout class; tilesM/tilesN of a descriptor must use this shape.
 int gemm_variant();
 void gemm_tile_shape(int cls, int *bm, int *bn);
 bool gemm_uses_3m(int cls);  // 3 DMMA products per complex MAC for this layout class
+int gemm_warps_per_tile(int cls);  // fused-dot partial sums per tile (one per consumer warp)
 int gemm_kernel_class(int layout_cls, int Ko);  // the launch class of a descriptor
 bool gemm_fused_dot_ok();    // the selected persistent GEMM has the fused-dot epilogue (4 warps/CTA)
 
 // Grouped launches: descs in device memory (all of one layout class); grid covers the tiles.
 cudaError_t launch_gemm_group(const GemmBatch *b, long long total_tiles, int cls, cudaStream_t st);
+cudaError_t launch_gemm_tma_group(const GemmTmaBatch *b, long long total_tiles, int cls, cudaStream_t st);
 // cls 0: a warp per dot and slice (modes 2, 3); cls 1: a CTA per dot and slice (modes 0, 1).
 // total_ctas = Σ Lt over the batch (one work item per dot and slice).
 inline int dot_class(int mode) { return mode == 0 || mode == 1 ? 1 : 0; }

@@ -58,7 +58,7 @@ class micco_stats(ctypes.Structure):
                 ("enqueue_ms", ctypes.c_double), ("host_pinned", ctypes.c_int32), ("gemm_3m", ctypes.c_int32),
                 ("gemm_dmma_flops", ctypes.c_double), ("dot_main_ms", ctypes.c_double),
                 ("dot_main_bytes", ctypes.c_double), ("dot_main_launches", ctypes.c_int64),
-                ("plan_ms", ctypes.c_double)]
+                ("plan_ms", ctypes.c_double), ("gemm_tma_launches", ctypes.c_int64)]
 
     def as_dict(self) -> Dict:
         d = {}
