@@ -921,14 +921,22 @@ __device__ __forceinline__ void zgemm_tma_body(const GemmTmaBatch &b, long long 
       const double2 a = as[i * 32];
       fa[buf][i][0] = a.x;
       fa[buf][i][1] = a.y;
+#ifdef TM_NO_SUMS
+      fa[buf][i][2] = a.x;  // (timing experiment only: wrong results)
+#else
       fa[buf][i][2] = a.x + a.y;  // Ar + Ai
+#endif
     }
 #pragma unroll
     for (int j = 0; j < NJ; ++j) {
       const double2 v = bs[j * 32];
       fb[buf][j][0] = v.x;
       fb[buf][j][1] = v.y;
+#ifdef TM_NO_SUMS
+      fb[buf][j][2] = v.y;
+#else
       fb[buf][j][2] = v.x + v.y;  // Br + Bi
+#endif
     }
   };
 
