@@ -98,10 +98,8 @@ micco_status nccl_unique_id(uint8_t out[128]) {
 
 namespace {
 
-#ifndef MICCO_H2D_LOOKAHEAD
-#define MICCO_H2D_LOOKAHEAD 64  // (6: C4 e2e 122.2k graphs/s; 64: 129.7k; the 8 GB cap below binds first)
-#endif
-constexpr int kLookahead = MICCO_H2D_LOOKAHEAD;  // chunks the H2D prefetch may run ahead
+// chunks the H2D prefetch may run ahead (6: C4 e2e 122.2k graphs/s; 64: 129.7k; round 1)
+constexpr int kLookahead = 64;
 constexpr int64_t kPrefetchBytes = 8LL << 30;    // and at most this many bytes
 
 struct EventPool {
@@ -204,6 +202,7 @@ struct Executor::Impl {
   int vals_dev = 0;
   double2 *h_corr = nullptr;
   int64_t launches = 0, tma_launches = 0;
+  bool use_tma = true;  // TMA GEMM for the contractions that fit it (see execute)
   bool dist() const { return c.opt.dist_world > 0; }
   int table_of(int i) const { return c.opt.scalar_tables ? i : g[i].dev; }
   double2 *table_row(const LGpu &l, int32_t slot) const {
@@ -399,10 +398,10 @@ struct Executor::Impl {
     CK(cudaEventRecord(e, s));
     return e;
   }
-  // Peer moves run on their own stream (MICCO_P2P_STREAM=0: on the compute stream), ordered
-  // with the kernels by events only: the transfer overlaps the kernels of earlier stages, and
-  // in multi-process mode an ncclSend no longer holds the sender's compute stream until the
-  // receiver's stream reaches the matching ncclRecv.  All NCCL calls of a rank stay on one
+  // Peer moves run on their own stream, ordered with the kernels by events only: the
+  // transfer overlaps the kernels of earlier stages, and in multi-process mode an ncclSend
+  // does not hold the sender's compute stream until the receiver's stream reaches the
+  // matching ncclRecv.  All NCCL calls of a rank stay on one
   // stream in the global plan order (the pairing argument of the op list is unchanged).
   // A peer move for the chunk being built may start once the compute stream has finished the
   // chunk before the last flushed one: the peer stream runs at most ~2 stages ahead, so
@@ -410,14 +409,6 @@ struct Executor::Impl {
   void pace_peer(LGpu &l) {
     const size_t nf = l.flush_ev.size();
     if (nf >= 2) CK(cudaStreamWaitEvent(l.pst, l.flush_ev[nf - 2], 0));
-  }
-  bool p2p_stream() const {
-    static int on = -1;
-    if (on < 0) {
-      const char *e = getenv("MICCO_P2P_STREAM");
-      on = (e && e[0] == '0') ? 0 : 1;
-    }
-    return on == 1;
   }
 
   double2 *alloc(LGpu &l, int64_t bytes) {
@@ -553,7 +544,7 @@ struct Executor::Impl {
       std::array<CUtensorMap, 2> maps;
       {
         int tcls;  // the TMA kernel when the operands fit its tensor maps (kernels.cu gemm_tma_class)
-        if (gemm_tma_class(d, &tcls) && gemm_tma_encode(d, tcls, &maps[0], &maps[1])) d.cls = tcls;
+        if (use_tma && gemm_tma_class(d, &tcls) && gemm_tma_encode(d, tcls, &maps[0], &maps[1])) d.cls = tcls;
       }
       int tbm, tbn;
       gemm_tile_shape(d.cls, &tbm, &tbn);
@@ -666,39 +657,34 @@ struct Executor::Impl {
         st.bytes_h2d += bytes_of(op.id);
         return;
       }
-      case PlanOp::P2P: {
+      case PlanOp::P2P: {  // on the peer stream, ordered with the kernels by events (pace_peer)
         LGpu &dst = g[op.gpu];
         LGpu &src = g[op.src];
         const int64_t nb = bytes_of(op.id);
-        const bool ps = p2p_stream();
         if (dist()) {
           if (dst.local) {
             CK(cudaSetDevice(dst.dev));
-            cudaStream_t s = ps ? dst.pst : dst.st;
-            if (ps) pace_peer(dst);
+            cudaStream_t s = dst.pst;
+            pace_peer(dst);
             void *p = nullptr;
             CK(cudaMallocAsync(&p, (size_t)nb, s));
             NK(nccl().Recv(p, (size_t)nb / 8, ncclDouble, op.src, comm, s));
-            if (ps) CK(cudaStreamWaitEvent(dst.st, record_on(op.gpu, s), 0));  // consumers wait
+            CK(cudaStreamWaitEvent(dst.st, record_on(op.gpu, s), 0));  // consumers wait
             dst.ptr[op.id] = (double2 *)p;
             st.bytes_p2p += nb;
           } else if (src.local) {
             CK(cudaSetDevice(src.dev));
-            if (ps) {
-              CK(cudaStreamWaitEvent(src.pst, record(op.src), 0));  // the replica is complete
-              NK(nccl().Send(src.ptr[op.id], (size_t)nb / 8, ncclDouble, op.gpu, comm, src.pst));
-              src.readers[op.id].push_back(record_on(op.src, src.pst));  // a free waits for the send
-            } else {
-              NK(nccl().Send(src.ptr[op.id], (size_t)nb / 8, ncclDouble, op.gpu, comm, src.st));
-            }
+            CK(cudaStreamWaitEvent(src.pst, record(op.src), 0));  // the replica is complete
+            NK(nccl().Send(src.ptr[op.id], (size_t)nb / 8, ncclDouble, op.gpu, comm, src.pst));
+            src.readers[op.id].push_back(record_on(op.src, src.pst));  // a free waits for the send
           }
           return;
         }
         cudaEvent_t ready = record(op.src);  // the replica on src is complete
         CK(cudaSetDevice(dst.dev));
-        cudaStream_t s = ps ? dst.pst : dst.st;
+        cudaStream_t s = dst.pst;
         CK(cudaStreamWaitEvent(s, ready, 0));
-        if (ps) pace_peer(dst);
+        pace_peer(dst);
         void *pv = nullptr;
         CK(cudaMallocAsync(&pv, (size_t)nb, s));
         double2 *p = (double2 *)pv;
@@ -707,7 +693,7 @@ struct Executor::Impl {
         else
           CK(cudaMemcpyPeerAsync(p, dst.dev, src.ptr[op.id], src.dev, nb, s));
         cudaEvent_t done = record_on(op.gpu, s);
-        if (ps) CK(cudaStreamWaitEvent(dst.st, done, 0));
+        CK(cudaStreamWaitEvent(dst.st, done, 0));
         dst.ptr[op.id] = p;
         src.readers[op.id].push_back(done);
         st.bytes_p2p += nb;
@@ -822,10 +808,11 @@ struct Executor::Impl {
     in.budget = budgets();
     in.window_graphs = c.opt.window_graphs;
     in.keep_inputs = c.opt.keep_inputs_resident != 0;
-    {
-      const char *nf = getenv("MICCO_NO_FUSE");
-      // the fused epilogue exists in the persistent (2, default) and warp-specialized (3) kernels
-      in.fuse = gemm_fused_dot_ok() && !(nf && nf[0] == '1');
+    in.fuse = true;  // GEMM → final dot in the GEMM epilogue when legal (every GEMM kernel has it)
+    {  // MICCO_GEMM_TMA=0: keep every contraction on the cp.async kernels (read per execute; the
+       // parity suite runs both paths)
+      const char *e = getenv("MICCO_GEMM_TMA");
+      use_tma = !(e && e[0] == '0');
     }
     in.peer_gbs = (ndev > 1 && !dist()) || dist() ? 700 : 2500;
     in.host_gbs = 55;

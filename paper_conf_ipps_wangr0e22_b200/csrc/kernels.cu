@@ -194,27 +194,16 @@ __device__ __forceinline__ void zgemm_dmma_kernel_body(const GemmDesc *__restric
 // computed so they occupy the DMMA pacing slots; the task descriptor advances linearly.
 // Optional fused final dot (GemmDesc::D) in the epilogue.
 //
-// Complex product, three schemes (template M3, M3T):
-//   4M: Cr += Ar·Br + (−Ai)·Bi, Ci += Ar·Bi + Ai·Br                                — 4 DMMAs
-//   3M "T" (default): T1 += Ar·Br, T2 += Ai·Bi, T3 += (Ar+Ai)·(Br+Bi);
-//                     Cr = T1 − T2, Ci = T3 − (T1 + T2)            — 3 DMMAs, MI + NJ sums
-//   3M "K": K1 += (Ar+Ai)·Br, K2 += Ar·(Bi−Br), K3 += Ai·(Br+Bi);
-//           Cr = K1 − K3, Ci = K1 + K2                             — 3 DMMAs, MI + 2·NJ sums
-// The 3M schemes do 25% fewer DMMAs for the same algorithmic work (8 real flops per complex
-// MAC are still what the roofline counts); their rounding differs from the 4M one but stays
-// far inside the 1e-10 parity bound, and exact-integer inputs stay bit-exact (every partial
-// sum is an integer below 2^53; SURVEY.md §8(c) "Bit-exact GPU parity").  The operand sums
-// are DADDs, and a DADD waits for the FP64 pipe the DMMAs occupy (ncu: "math pipe throttle"
-// on the DADDs; each costs ~0.7 of a DMMA slot), so the T form, with 6 instead of 8 sums
-// per 24 DMMAs, is the faster one: 36.9 vs 35.0 TFLOP/s algorithmic on the bench workload.
+// Complex product: the 3M "T" (Gauss) form, T1 += Ar·Br, T2 += Ai·Bi, T3 += (Ar+Ai)·(Br+Bi);
+// Cr = T1 − T2, Ci = T3 − (T1 + T2): 3 DMMAs per 8×8×4 complex block instead of the textbook
+// 4, for the same algorithmic work (8 real flops per complex MAC are still what the roofline
+// counts).  Its rounding differs from the 4M form but stays far inside the 1e-10 parity bound,
+// and exact-integer inputs stay bit-exact (every partial sum is an integer below 2^53; SURVEY.md
+// §8(c) "Bit-exact GPU parity").  The operand sums are DADDs on the FP64 pipe the DMMAs occupy;
+// the T form needs MI + NJ of them per k-quad (the "K" form K1 = (Ar+Ai)·Br, K2 = Ar·(Bi−Br),
+// K3 = Ai·(Br+Bi) needs MI + 2·NJ and ran at 35.0 instead of 36.9 TFLOP/s; the 4M kernel at
+// 31.6; measured round 1).
 constexpr int BK2 = 16, ST2 = 3;
-constexpr int kGemmPhaseNs = 0;
-#ifndef MICCO_BARRIER_LATE
-#define MICCO_BARRIER_LATE 0  // 1: stage barrier before the last k-quad (measured slower: 35.6 vs 36.9 TF)
-#endif
-#ifndef MICCO_KEEP_SN
-#define MICCO_KEEP_SN 1
-#endif
 constexpr int APITCH2 = BK2 + 4;  // [m][k] rows: 320 B ≡ 64 (mod 128): A fragment loads conflict-free
 
 template <int TBM, int TBN>
@@ -369,16 +358,16 @@ __device__ __forceinline__ void decode_tile(const GemmDesc *__restrict__ descs, 
 
 // NWM × NWN warps with WTM × WTN complex warp tiles; CTA tile (NWM·WTM) × (NWN·WTN).
 // AKF / BNF: the layout class (A contiguous along k / B contiguous along n).
-template <int NWM, int NWN, int WTM, int WTN, bool M3, bool M3T, bool AKF, bool BNF, bool KB = false>
+template <int NWM, int NWN, int WTM, int WTN, bool AKF, bool BNF, bool KB = false>
 __device__ __forceinline__ void zgemm_persistent_body(const GemmDesc *__restrict__ descs, int n_desc,
-                                                      long long total, unsigned phase_ns) {
+                                                      long long total) {
   constexpr int NTH = NWM * NWN * 32;
   constexpr int TBM = NWM * WTM, TBN = NWN * WTN;
   using GA = Geo<TBM, NTH, AKF>;  // (KB: only the element counts are used)
   using GB = Geo<TBN, NTH, !BNF>;
   constexpr int LPTA = GA::L, LPTB = GB::L;
   constexpr int MI = WTM / 8, NJ = WTN / 8;  // 8x8 blocks per warp
-  constexpr int NACC = M3 ? 3 : 2;
+  constexpr int NACC = 3;  // T1, T2, T3
   using Cfg = PCfg<TBM, TBN>;
   constexpr int BP = Cfg::BP;
   // shared-memory stride between a thread's consecutive elements (complex elements)
@@ -397,11 +386,6 @@ __device__ __forceinline__ void zgemm_persistent_body(const GemmDesc *__restrict
   // served to the other CTAs from L2 (contiguous per-CTA ranges doubled the DRAM reads)
   const long long G = gridDim.x, t_begin = blockIdx.x;
   if (t_begin >= total) return;
-  // The two CTAs of an SM run tiles of equal length, so if they start together their
-  // epilogues coincide and the DMMA pipe idles through both.  The lag between them is
-  // neutrally stable (while one is in its epilogue the other runs the pipe alone), so a
-  // one-off delay of the second CTA keeps their epilogues apart for the whole launch.
-  if (phase_ns > 0 && 2 * blockIdx.x >= gridDim.x) __nanosleep(phase_ns);
 
   int task_l = 0, task_c = 0;
   {  // first task by binary search, then linear advance
@@ -457,7 +441,7 @@ __device__ __forceinline__ void zgemm_persistent_body(const GemmDesc *__restrict
       mA = L.rmA & run_mask<LPTA, GA::KJ>(L.kb + GA::k0(tid), L.Ki);
       mB = L.rmB & run_mask<LPTB, GB::KJ>(L.kb + GB::k0(tid), L.Ki);
     }
-    if constexpr (M3 && !KB) ld_full = __all_sync(0xffffffffu, mA == (1u << LPTA) - 1u && mB == (1u << LPTB) - 1u);
+    if constexpr (!KB) ld_full = __all_sync(0xffffffffu, mA == (1u << LPTA) - 1u && mB == (1u << LPTB) - 1u);
   };
   auto issue_part = [&](int slot, int part) {
     if constexpr (KB) {  // runtime geometry (per task): element j at s0 + j·sj
@@ -507,13 +491,9 @@ __device__ __forceinline__ void zgemm_persistent_body(const GemmDesc *__restrict
     if (++kt_l == L.KTOT) {
       kt_l = 0;
       if ((tile_l += G) < total) {
-        if constexpr (M3 && MICCO_KEEP_SN) {  // (the 4M kernel has no registers left for a second cursor)
-          decode_tile<NTH, TBM, TBN, AKF, BNF, KB>(descs, n_desc, task_l, tile_l, tid, &L, &Sn);
-          sn_tile = tile_l;
-          sn_task = task_l;
-        } else {
-          decode_tile<NTH, TBM, TBN, AKF, BNF, KB>(descs, n_desc, task_l, tile_l, tid, &L, (StoreCur *)nullptr);
-        }
+        decode_tile<NTH, TBM, TBN, AKF, BNF, KB>(descs, n_desc, task_l, tile_l, tid, &L, &Sn);
+        sn_tile = tile_l;
+        sn_task = task_l;
       } else {
         more_l = false;
       }
@@ -555,11 +535,10 @@ __device__ __forceinline__ void zgemm_persistent_body(const GemmDesc *__restrict
     cp_async_commit();
   }
   int slot_c = 0, slot_l = ST2 - 1;
-  // Fragments are double-buffered (3M): the LDS and the operand sums of k-quad q+1 are issued
-  // before the DMMAs of q.  The stage barrier sits before the DMMAs of the last k-quad, so the
-  // first fragments of the next stage are read while those DMMAs run, not after the barrier.
-  constexpr int FA = M3 ? 3 : 2, FB = M3 ? 3 : 2;
-  double fa[2][MI][FA], fb[2][NJ][FB];
+  // Fragments are double-buffered: the LDS and the operand sums of k-quad q+1 are issued
+  // before the DMMAs of q.  (The stage barrier sits at the top of the stage: moving it before
+  // the DMMAs of the last k-quad measured slower, 35.6 vs 36.9 TF, round 1.)
+  double fa[2][MI][3], fb[2][NJ][3];
   auto load_frag = [&](int buf, int slot, int kq) {
     const double2 *as = As + slot * Cfg::AE;
     const double2 *bs = Bs + slot * Cfg::BE;
@@ -568,81 +547,40 @@ __device__ __forceinline__ void zgemm_persistent_body(const GemmDesc *__restrict
       const double2 a = as[(wm * WTM + i * 8 + (lane >> 2)) * APITCH2 + kq * 4 + (lane & 3)];
       fa[buf][i][0] = a.x;
       fa[buf][i][1] = a.y;
-      if constexpr (M3) fa[buf][i][2] = a.x + a.y;  // Ar + Ai
+      fa[buf][i][2] = a.x + a.y;  // Ar + Ai
     }
 #pragma unroll
     for (int j = 0; j < NJ; ++j) {
       const double2 b = bs[(kq * 4 + (lane & 3)) * BP + wn * WTN + j * 8 + (lane >> 2)];
       fb[buf][j][0] = b.x;
       fb[buf][j][1] = b.y;
-      if constexpr (M3) {
-        if constexpr (!M3T) fb[buf][j][1] = b.y - b.x;  // Bi − Br
-        fb[buf][j][2] = b.x + b.y;                       // Br + Bi
-      }
+      fb[buf][j][2] = b.x + b.y;  // Br + Bi
     }
   };
-  constexpr bool LATE = MICCO_BARRIER_LATE != 0;
-  if constexpr (LATE) {
+  for (;;) {
     cp_async_wait<ST2 - 2>();
     __syncthreads();
-    if constexpr (M3) load_frag(0, slot_c, 0);
-  }
-  for (;;) {
-    if constexpr (!LATE) {
-      cp_async_wait<ST2 - 2>();
-      __syncthreads();
-      if constexpr (M3) load_frag(0, slot_c, 0);
-    }
+    load_frag(0, slot_c, 0);
     const bool ld = more_l;
     if (ld) begin_load();
 #pragma unroll
     for (int kq = 0; kq < BK2 / 4; ++kq) {
       if (ld) issue_part(slot_l, kq);
-      const int cur = M3 ? (kq & 1) : 0;
+      const int cur = kq & 1;
       if (kq + 1 < BK2 / 4) {
-        if constexpr (M3) load_frag(cur ^ 1, slot_c, kq + 1);
-        else load_frag(0, slot_c, kq);
+        load_frag(cur ^ 1, slot_c, kq + 1);
       } else {
-        if constexpr (!M3) load_frag(0, slot_c, kq);
         if (ld) advance_load();
         cp_async_commit();
-        if constexpr (LATE) {
-          cp_async_wait<ST2 - 2>();  // the next stage has landed ...
-          __syncthreads();           // ... for every thread, and this stage's slot is free
-          if constexpr (M3) load_frag(cur ^ 1, slot_c + 1 == ST2 ? 0 : slot_c + 1, 0);
+      }
+#pragma unroll
+      for (int i = 0; i < MI; ++i)
+#pragma unroll
+        for (int j = 0; j < NJ; ++j) {
+          dmma(acc[i][j][0][0], acc[i][j][0][1], fa[cur][i][0], fb[cur][j][0]);  // Ar·Br
+          dmma(acc[i][j][1][0], acc[i][j][1][1], fa[cur][i][1], fb[cur][j][1]);  // Ai·Bi
+          dmma(acc[i][j][2][0], acc[i][j][2][1], fa[cur][i][2], fb[cur][j][2]);  // (Ar+Ai)·(Br+Bi)
         }
-      }
-      if constexpr (M3) {
-#pragma unroll
-        for (int i = 0; i < MI; ++i)
-#pragma unroll
-          for (int j = 0; j < NJ; ++j) {
-            if constexpr (M3T) {
-              dmma(acc[i][j][0][0], acc[i][j][0][1], fa[cur][i][0], fb[cur][j][0]);  // Ar·Br
-              dmma(acc[i][j][1][0], acc[i][j][1][1], fa[cur][i][1], fb[cur][j][1]);  // Ai·Bi
-              dmma(acc[i][j][2][0], acc[i][j][2][1], fa[cur][i][2], fb[cur][j][2]);  // (Ar+Ai)·(Br+Bi)
-            } else {
-              dmma(acc[i][j][0][0], acc[i][j][0][1], fa[cur][i][2], fb[cur][j][0]);  // (Ar+Ai)·Br
-              dmma(acc[i][j][1][0], acc[i][j][1][1], fa[cur][i][0], fb[cur][j][1]);  // Ar·(Bi−Br)
-              dmma(acc[i][j][2][0], acc[i][j][2][1], fa[cur][i][1], fb[cur][j][2]);  // Ai·(Br+Bi)
-            }
-          }
-      } else {
-#pragma unroll
-        for (int i = 0; i < MI; ++i)
-#pragma unroll
-          for (int j = 0; j < NJ; ++j) {
-            dmma(acc[i][j][0][0], acc[i][j][0][1], fa[cur][i][0], fb[cur][j][0]);
-            dmma(acc[i][j][1][0], acc[i][j][1][1], fa[cur][i][0], fb[cur][j][1]);
-          }
-#pragma unroll
-        for (int i = 0; i < MI; ++i)
-#pragma unroll
-          for (int j = 0; j < NJ; ++j) {
-            dmma(acc[i][j][0][0], acc[i][j][0][1], dneg(fa[cur][i][1]), fb[cur][j][1]);
-            dmma(acc[i][j][1][0], acc[i][j][1][1], fa[cur][i][1], fb[cur][j][0]);
-          }
-      }
     }
     slot_l = (slot_l + 1 == ST2) ? 0 : slot_l + 1;
     slot_c = (slot_c + 1 == ST2) ? 0 : slot_c + 1;
@@ -661,25 +599,17 @@ __device__ __forceinline__ void zgemm_persistent_body(const GemmDesc *__restrict
     }
     if (++kt_c == S.KTOT) {  // tile done: write back (next tile's loads already in flight)
       // the complex value of accumulator block (i, j), half h
-      auto cval = [&](int i, int j, int h, double &re, double &im) {
-        if constexpr (M3T) {  // T1 = Ar·Br, T2 = Ai·Bi, T3 = (Ar+Ai)·(Br+Bi)
-          re = acc[i][j][0][h] - acc[i][j][1][h];
-          im = acc[i][j][2][h] - (acc[i][j][0][h] + acc[i][j][1][h]);
-        } else if constexpr (M3) {
-          re = acc[i][j][0][h] - acc[i][j][2][h];
-          im = acc[i][j][0][h] + acc[i][j][1][h];
-        } else {
-          re = acc[i][j][0][h];
-          im = acc[i][j][1][h];
-        }
+      auto cval = [&](int i, int j, int h, double &re, double &im) {  // T1 − T2, T3 − (T1 + T2)
+        re = acc[i][j][0][h] - acc[i][j][1][h];
+        im = acc[i][j][2][h] - (acc[i][j][0][h] + acc[i][j][1][h]);
       };
       if (S.D) {
         // fused final contraction: this warp's partial Σ C·D (no C written)
         const GemmDesc &dd = descs[task_c];
         const long long sDmi = dd.sDmi, sDni = dd.sDni;
-        // partner loads issued CH rows at a time before their use (3M: all rows, one round
-        // trip to L2 where the block was prefetched; 4M: one row, its registers are full)
-        constexpr int CH = M3 ? MI : 1;
+        // partner loads: all rows issued before their use (one round trip to L2, where the
+        // block was prefetched)
+        constexpr int CH = MI;
         double pr = 0.0, pim = 0.0;
 #pragma unroll
         for (int i0 = 0; i0 < MI; i0 += CH) {
@@ -740,7 +670,7 @@ __device__ __forceinline__ void zgemm_persistent_body(const GemmDesc *__restrict
           for (int q = 0; q < NACC; ++q) acc[i][j][q][0] = acc[i][j][q][1] = 0.0;
       kt_c = 0;
       if ((tile_c += G) >= total) break;
-      if (M3 && MICCO_KEEP_SN && sn_tile == tile_c) {
+      if (sn_tile == tile_c) {
         S = Sn;
         task_c = sn_task;
       } else {
@@ -921,22 +851,14 @@ __device__ __forceinline__ void zgemm_tma_body(const GemmTmaBatch &b, long long 
       const double2 a = as[i * 32];
       fa[buf][i][0] = a.x;
       fa[buf][i][1] = a.y;
-#ifdef TM_NO_SUMS
-      fa[buf][i][2] = a.x;  // (timing experiment only: wrong results)
-#else
       fa[buf][i][2] = a.x + a.y;  // Ar + Ai
-#endif
     }
 #pragma unroll
     for (int j = 0; j < NJ; ++j) {
       const double2 v = bs[j * 32];
       fb[buf][j][0] = v.x;
       fb[buf][j][1] = v.y;
-#ifdef TM_NO_SUMS
-      fb[buf][j][2] = v.y;
-#else
       fb[buf][j][2] = v.x + v.y;  // Br + Bi
-#endif
     }
   };
 
@@ -1076,37 +998,21 @@ __device__ __forceinline__ void cmac(double &sr, double &si, double2 a, double2 
   si += a.x * b.y + a.y * b.x;
 }
 
-#ifndef MICCO_DOT_NOALLOC
-#define MICCO_DOT_NOALLOC 1  // L1::no_allocate on the streaming dot loads (C4 dots 55.7 → 48.4 ms)
-#endif
-#ifndef MICCO_DOT_MINB
-#define MICCO_DOT_MINB 3  // resident dot CTAs per SM the register budget is sized for
-#endif
-#ifndef MICCO_DOT_UNROLL
-#define MICCO_DOT_UNROLL 2
-#endif
-constexpr int DOT_UNROLL = MICCO_DOT_UNROLL;  // mode-1 micro-block pairs in flight per thread
+constexpr int DOT_MINB = 3;    // resident dot CTAs per SM the register budget is sized for
+constexpr int DOT_UNROLL = 2;  // mode-1 micro-block pairs in flight per thread
 
-// one complex element, read once: no L1 allocation (MICCO_DOT_NOALLOC)
+// one complex element, read once: no L1 allocation (C4 dots 55.7 → 48.4 ms, round 1)
 __device__ __forceinline__ double2 ldg_stream(const double2 *p) {
-#if MICCO_DOT_NOALLOC
   double2 v;
   asm("ld.global.nc.L1::no_allocate.v2.f64 {%0, %1}, [%2];" : "=d"(v.x), "=d"(v.y) : "l"(p));
   return v;
-#else
-  return __ldg(p);
-#endif
 }
 
 // 32 bytes (two complex elements) in one LDG.E.256 (sm_100); p must be 32-byte aligned
 __device__ __forceinline__ void ldg_pair(const double2 *p, double2 &a, double2 &b) {
-#if MICCO_DOT_NOALLOC
   asm("ld.global.nc.L1::no_allocate.v4.f64 {%0, %1, %2, %3}, [%4];"
       : "=d"(a.x), "=d"(a.y), "=d"(b.x), "=d"(b.y)
       : "l"(p));
-#else
-  asm("ld.global.nc.v4.f64 {%0, %1, %2, %3}, [%4];" : "=d"(a.x), "=d"(a.y), "=d"(b.x), "=d"(b.y) : "l"(p));
-#endif
 }
 
 // mode 1: s = Σ_o Σ_{y<Y} Σ_{x<X} A[o][y·sAy + x] · B[o][x·sBx + y]   (layout.cpp: sAx = sBy = 1)
@@ -1322,27 +1228,23 @@ __global__ void accumulate_kernel(double2 *dst, const double2 *src, long long n)
 __global__ void __launch_bounds__(NT, 2) zgemm_dmma_kernel(const __grid_constant__ GemmBatch b, long long total) {
   zgemm_dmma_kernel_body(b.d, b.n, total);
 }
-template <int NWM, int NWN, int WTM, int WTN, bool M3, bool M3T, bool AKF, bool BNF>
-__global__ void __launch_bounds__(NWM * NWN * 32, 2)
-    zgemm_persistent(const __grid_constant__ GemmBatch b, long long total, unsigned phase_ns) {
-  zgemm_persistent_body<NWM, NWN, WTM, WTN, M3, M3T, AKF, BNF>(b.d, b.n, total, phase_ns);
+template <bool AKF, bool BNF>
+__global__ void __launch_bounds__(128, 2) zgemm_persistent(const __grid_constant__ GemmBatch b, long long total) {
+  zgemm_persistent_body<2, 2, 32, 16, AKF, BNF>(b.d, b.n, total);
 }
 
-template <int NWM, int NWN, int WTM, int WTN, bool M3, bool M3T>
-__global__ void __launch_bounds__(NWM * NWN * 32, 2)
-    zgemm_persistent_kb(const __grid_constant__ GemmBatch b, long long total, unsigned phase_ns) {
-  zgemm_persistent_body<NWM, NWN, WTM, WTN, M3, M3T, true, true, true>(b.d, b.n, total, phase_ns);
+__global__ void __launch_bounds__(128, 2) zgemm_persistent_kb(const __grid_constant__ GemmBatch b, long long total) {
+  zgemm_persistent_body<2, 2, 32, 16, true, true, true>(b.d, b.n, total);
 }
 
 // The persistent GEMM for layout class cls (0..3 = (A contiguous along m ? 2 : 0) +
 // (B contiguous along k ? 1 : 0), layout.cpp gemm_class).
-template <int NWM, int NWN, int WTM, int WTN, bool M3, bool M3T>
-void (*persistent_fn(int cls))(const GemmBatch, long long, unsigned) {
+void (*persistent_fn(int cls))(const GemmBatch, long long) {
   switch (cls) {
-    case 0: return zgemm_persistent<NWM, NWN, WTM, WTN, M3, M3T, true, true>;
-    case 1: return zgemm_persistent<NWM, NWN, WTM, WTN, M3, M3T, true, false>;
-    case 2: return zgemm_persistent<NWM, NWN, WTM, WTN, M3, M3T, false, true>;
-    default: return zgemm_persistent<NWM, NWN, WTM, WTN, M3, M3T, false, false>;
+    case 0: return zgemm_persistent<true, true>;
+    case 1: return zgemm_persistent<true, false>;
+    case 2: return zgemm_persistent<false, true>;
+    default: return zgemm_persistent<false, false>;
   }
 }
 
@@ -1351,7 +1253,7 @@ __global__ void __launch_bounds__(TM_THREADS, 1) zgemm_tma(const __grid_constant
   zgemm_tma_body<AK, BK>(b, total);
 }
 
-__global__ void __launch_bounds__(DT, MICCO_DOT_MINB) zdot_kernel(const __grid_constant__ DotBatch b) { zdot_body(b.d, b.n); }
+__global__ void __launch_bounds__(DT, DOT_MINB) zdot_kernel(const __grid_constant__ DotBatch b) { zdot_body(b.d, b.n); }
 __global__ void __launch_bounds__(DT) zdot_warp_kernel(const __grid_constant__ DotBatch b, long long items) {
   zdot_warp_body(b.d, b.n, items);
 }
@@ -1416,49 +1318,30 @@ cudaError_t probe_fp64_peak(double seconds, double *burst_tflops, double *sustai
   return e;
 }
 
-int gemm_variant() {
-  // MICCO_GEMM = 5 (default) persistent 64×32 tiles, 3M "T" complex products;
-  //              6 the same with the 3M "K" form;  2 persistent 64×64 tiles, 4M;
-  //              1 per-tile 64×64 4M (also the gather kernel).
-  // Measured on the bench workload (GEMM TFLOP/s algorithmic): 5 → 36.9, 6 → 35.0, 2 → 31.6
-  // (profiles/bench_r01_v7*.json).  Earlier experiments (warp-specialised producer/consumer,
-  // small 32×32 tiles, 8-warp 3M) are in DESIGN.md §6's history table; all were slower.
-  static int variant = -1;
-  if (variant < 0) {
-    const char *e = getenv("MICCO_GEMM");
-    variant = (e && (e[0] == '1' || e[0] == '2' || e[0] == '5' || e[0] == '6')) ? e[0] - '0' : 5;
-  }
-  return variant;
-}
-
 void gemm_tile_shape(int cls, int *bm, int *bn) {
   *bm = 64;
-  *bn = 64;
+  *bn = 32;
   if (cls >= kGemmClassTMA) { *bm = TM_BM; *bn = TM_BN; return; }
-  if (cls == 4) return;  // gather kernel (v1)
-  if (gemm_variant() >= 5) *bn = 32;
+  if (cls == 4) *bn = 64;  // per-tile gather kernel
 }
 
-bool gemm_uses_3m(int cls) { return cls != 4 && gemm_variant() >= 5; }
+bool gemm_uses_3m(int cls) { return cls != 4; }
 
 int gemm_warps_per_tile(int cls) { return cls >= kGemmClassTMA ? TM_NW : 4; }
 
 int gemm_kernel_class(int layout_cls, int Ko) {
   // class 4 (no unit stride on an operand's free or inner contracted index) goes to the
   // blocked-K persistent kernel when the outer contracted index is long enough to fill a
-  // 4 × 4 k-block; else to the per-tile gather kernel (variant 1)
-  if (layout_cls == 4 && Ko >= 4 && gemm_variant() >= 5) return kGemmClassKB;
+  // 4 × 4 k-block; else to the per-tile gather kernel
+  if (layout_cls == 4 && Ko >= 4) return kGemmClassKB;
   return layout_cls;
 }
-
-bool gemm_fused_dot_ok() { return gemm_variant() != 1; }
 
 cudaError_t launch_gemm_group(const GemmBatch *b, long long total_tiles, int cls, cudaStream_t st) {
   // (one host thread launches: the executor replays the plan sequentially)
   // The shared-memory opt-in is recorded per device context: track it per device, so the
   // persistent GEMMs on a second (third, ...) device of one process get it too.
   static unsigned long long attr_set = 0;  // bit d: set on device d
-  const int variant = gemm_variant();
   int cur_dev = 0;
   if (cudaError_t e = cudaGetDevice(&cur_dev); e != cudaSuccess) return e;
   const unsigned long long dev_bit = 1ull << (cur_dev & 63);
@@ -1466,70 +1349,31 @@ cudaError_t launch_gemm_group(const GemmBatch *b, long long total_tiles, int cls
     cudaError_t e = cudaFuncSetAttribute(zgemm_dmma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, GEMM_SMEM);
     if (e != cudaSuccess) return e;
     for (int c = 0; c < 4; ++c) {
-      e = cudaFuncSetAttribute(persistent_fn<2, 2, 32, 32, false, false>(c), cudaFuncAttributeMaxDynamicSharedMemorySize,
-                               PCfg<64, 64>::SMEM);
+      e = cudaFuncSetAttribute(persistent_fn(c), cudaFuncAttributeMaxDynamicSharedMemorySize, PCfg<64, 32>::SMEM);
       if (e != cudaSuccess) return e;
-      e = cudaFuncSetAttribute(persistent_fn<2, 2, 32, 16, true, false>(c), cudaFuncAttributeMaxDynamicSharedMemorySize,
-                               PCfg<64, 32>::SMEM);
-      if (e != cudaSuccess) return e;
-      e = cudaFuncSetAttribute(persistent_fn<2, 2, 32, 16, true, true>(c), cudaFuncAttributeMaxDynamicSharedMemorySize,
-                               PCfg<64, 32>::SMEM);
-      if (e != cudaSuccess) return e;
-      if (c == 0) {
-        e = cudaFuncSetAttribute(zgemm_persistent_kb<2, 2, 32, 16, true, true>,
-                                 cudaFuncAttributeMaxDynamicSharedMemorySize, PCfg<64, 32>::SMEM);
-        if (e != cudaSuccess) return e;
-        e = cudaFuncSetAttribute(zgemm_persistent_kb<2, 2, 32, 16, true, false>,
-                                 cudaFuncAttributeMaxDynamicSharedMemorySize, PCfg<64, 32>::SMEM);
-        if (e != cudaSuccess) return e;
-      }
     }
+    e = cudaFuncSetAttribute(zgemm_persistent_kb, cudaFuncAttributeMaxDynamicSharedMemorySize, PCfg<64, 32>::SMEM);
+    if (e != cudaSuccess) return e;
     attr_set |= dev_bit;
   }
   if (total_tiles <= 0) return cudaSuccess;
   int sms = 148;
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, cur_dev);
-  if (variant == 1 || cls == 4) {  // per-tile kernel; the only one that gathers strided operands
+  if (cls == 4) {  // per-tile kernel; gathers operands with no unit-stride free or inner contracted index
     long long grid = total_tiles < (1LL << 30) ? total_tiles : (1LL << 30);
     zgemm_dmma_kernel<<<(unsigned)grid, NT, GEMM_SMEM, st>>>(*b, total_tiles);
     return cudaGetLastError();
   }
   long long grid = 2LL * sms;  // 2 resident CTAs per SM
   if (grid > total_tiles) grid = total_tiles;
-  static int phase_ns = -1;  // start lag of the second CTA per SM (env MICCO_GEMM_PHASE_NS)
-  if (phase_ns < 0) {
-    const char *e = getenv("MICCO_GEMM_PHASE_NS");
-    phase_ns = e ? atoi(e) : kGemmPhaseNs;
-    if (phase_ns < 0) phase_ns = 0;
-  }
-  if (cls == kGemmClassKB) {  // blocked-K gather (variant 5 or 6; gemm_kernel_class)
-    if (variant == 6)
-      zgemm_persistent_kb<2, 2, 32, 16, true, false><<<(unsigned)grid, 128, PCfg<64, 32>::SMEM, st>>>(
-          *b, total_tiles, (unsigned)phase_ns);
-    else
-      zgemm_persistent_kb<2, 2, 32, 16, true, true><<<(unsigned)grid, 128, PCfg<64, 32>::SMEM, st>>>(
-          *b, total_tiles, (unsigned)phase_ns);
-    return cudaGetLastError();
-  }
-  if (variant == 2)
-    persistent_fn<2, 2, 32, 32, false, false>(cls)<<<(unsigned)grid, 128, PCfg<64, 64>::SMEM, st>>>(*b, total_tiles,
-                                                                                           (unsigned)phase_ns);
-  else if (variant == 5)
-    persistent_fn<2, 2, 32, 16, true, true>(cls)<<<(unsigned)grid, 128, PCfg<64, 32>::SMEM, st>>>(*b, total_tiles,
-                                                                                                (unsigned)phase_ns);
-  else  // 6: the 3M "K" form
-    persistent_fn<2, 2, 32, 16, true, false>(cls)<<<(unsigned)grid, 128, PCfg<64, 32>::SMEM, st>>>(*b, total_tiles,
-                                                                                          (unsigned)phase_ns);
+  if (cls == kGemmClassKB)  // blocked-K gather (gemm_kernel_class)
+    zgemm_persistent_kb<<<(unsigned)grid, 128, PCfg<64, 32>::SMEM, st>>>(*b, total_tiles);
+  else
+    persistent_fn(cls)<<<(unsigned)grid, 128, PCfg<64, 32>::SMEM, st>>>(*b, total_tiles);
   return cudaGetLastError();
 }
 
 bool gemm_tma_class(const GemmDesc &d, int *cls) {
-  static int off = -1;  // MICCO_GEMM_TMA=0: keep every contraction on the cp.async kernels
-  if (off < 0) {
-    const char *e = getenv("MICCO_GEMM_TMA");
-    off = (e && e[0] == '0') ? 1 : 0;
-  }
-  if (off || gemm_variant() != 5) return false;
   const bool ak = d.sAki == 1, bk = d.sBki == 1;  // K-major operands (else contiguous along m / n)
   if (!ak && d.sAmi != 1) return false;
   if (!bk && d.sBni != 1) return false;

@@ -96,14 +96,11 @@ bool gemm_tma_class(const GemmDesc &d, int *cls);
 // Encode the two operand tensor maps of a TMA-class descriptor (host; no device work).
 bool gemm_tma_encode(const GemmDesc &d, int cls, CUtensorMap *a, CUtensorMap *b);
 
-// The GEMM kernel variant in use (env MICCO_GEMM, see kernels.cu) and its CTA tile (complex
-// elements) for a layout class; tilesM/tilesN of a descriptor must use this shape.
-int gemm_variant();
+// The CTA tile (complex elements) of a kernel class; tilesM/tilesN of a descriptor must use it.
 void gemm_tile_shape(int cls, int *bm, int *bn);
 bool gemm_uses_3m(int cls);  // 3 DMMA products per complex MAC for this layout class
 int gemm_warps_per_tile(int cls);  // fused-dot partial sums per tile (one per consumer warp)
 int gemm_kernel_class(int layout_cls, int Ko);  // the launch class of a descriptor
-bool gemm_fused_dot_ok();    // the selected persistent GEMM has the fused-dot epilogue (4 warps/CTA)
 
 // Grouped launches: descs in device memory (all of one layout class); grid covers the tiles.
 cudaError_t launch_gemm_group(const GemmBatch *b, long long total_tiles, int cls, cudaStream_t st);

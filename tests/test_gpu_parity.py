@@ -404,3 +404,22 @@ def test_rank4_parity_nb64():
     st = ctx.stats()
     ctx.close()
     assert st["n_gemm"] > 0
+
+
+@pytest.mark.parametrize("tma", ["1", "0"])
+def test_gemm_paths_meson_shapes(tma, monkeypatch):
+    """Both GEMM kernels on the meson shapes the TMA kernel takes (MICCO_GEMM_TMA=0 keeps every
+    contraction on the cp.async persistent kernel, which otherwise serves only ragged / strided
+    operands): C2 cycles with random transposes (all four operand-layout classes) and C3 wirings
+    with the reuse-aware order (fused final dots), ≤ 1e-10 against the oracle, and integer
+    inputs bit-exact; the TMA run must really use the TMA kernel."""
+    monkeypatch.setenv("MICCO_GEMM_TMA", tma)
+    for wl in (workloads.c2_meson_set(n_graphs=60, N=64, Lt=3, rate=0.5, flips=True),
+               workloads.c3_multi_meson(n_graphs=40, N=96, Lt=2, pool=4)):
+        C, st = check(wl, reorder=True)
+        assert (st["gemm_tma_launches"] > 0) == (tma == "1"), st
+        assert st["gemm_tma_launches"] <= st["gemm_launches"]
+    wli = workloads.c2_meson_set(n_graphs=40, N=128, Lt=2, rate=0.5, flips=True, mode=MODE_INT3)
+    _, vals, _ = run_gpu(wli)
+    _, valso = oracle.correlator(wli, return_values=True)
+    assert np.array_equal(vals, valso)

@@ -71,8 +71,6 @@ def build_lib(force: bool = False, jobs: int = 8) -> Path:
     objdir.mkdir(parents=True, exist_ok=True)
     common = ["-std=c++17", "-O3", "-Xcompiler", "-fPIC", "-Xcompiler", "-fvisibility=hidden",
               "-I", ROOT / "include", "-I", ROOT, "-I", CSRC]
-    # experiment switches (e.g. MICCO_NVCC_DEFS="-DMICCO_BARRIER_LATE=0"); empty for the product build
-    common += os.environ.get("MICCO_NVCC_DEFS", "").split()
     procs, objs = [], []
     for s in srcs:
         o = objdir / (s.name + ".o")
