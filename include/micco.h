@@ -225,6 +225,13 @@ typedef struct {
                                   replay when planning streams; sched_ms = the same) */
   int64_t gemm_tma_launches;   /* GEMM launches on the TMA warp-specialized kernel (the rest ran on
                                   the cp.async kernels: ragged k, odd rows, 6-D views) */
+  double model_s;              /* the plan's modelled time (planner cost model, core.h kModel*):
+                                  Σ over stages of max over GPUs of flops + host bytes + peer bytes
+                                  times (copies serialised with the kernels: pessimistic) */
+  double model_overlap_s;      /* the same with each GPU's copies overlapping its kernels:
+                                  Σ over stages of max over GPUs of max(flops, host, peer) time */
+  int64_t peak_bytes;          /* the plan's largest resident set on one GPU (its memory demand) */
+  int32_t window_graphs;       /* the window the plan used (options.window_graphs or the auto choice) */
 } micco_stats;
 
 MICCO_API micco_status micco_get_stats(const micco_ctx *ctx, micco_stats *out);
@@ -281,8 +288,8 @@ MICCO_API micco_status micco_plan_ops(micco_ctx *ctx, int32_t n_gpus, const int3
  * ceil(pairs/n_gpus), log2 mean operand bytes, repeated rate, resident rate, n_gpus, memory
  * pressure = max resident/budget; taken before the vector is scheduled) into features[6*s..]
  * and the bounds used into bounds[3*s..].  *n_stages receives the stage count, *predicted_s
- * the plan's modelled time (max over GPUs per stage of flops/30 TF/s + host bytes/55 GB/s +
- * peer bytes/700 GB/s, summed over stages).  Needs options.mem_budget_bytes; no GPU. */
+ * the plan's modelled time (max over GPUs per stage of flops/42.9 TF/s + host bytes/55.5 GB/s +
+ * peer bytes/770 GB/s, summed over stages; core.h kModel*).  Needs options.mem_budget_bytes; no GPU. */
 MICCO_API micco_status micco_plan_stages(micco_ctx *ctx, int32_t n_gpus, int32_t bound_mode,
                                          const int32_t *reuse_bound, int64_t max_stages,
                                          double *features, int32_t *bounds, int64_t *n_stages,

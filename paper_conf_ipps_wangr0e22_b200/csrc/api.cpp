@@ -322,9 +322,9 @@ Plan host_plan(Context &c, int32_t n_gpus, const int32_t *reuse_bound, int32_t b
   in.budget.assign(n_gpus, c.opt.mem_budget_bytes);
   in.window_graphs = c.opt.window_graphs;
   in.keep_inputs = c.opt.keep_inputs_resident != 0;
-  in.peer_gbs = 700;
-  in.host_gbs = 55;
-  in.flops_per_s = 30e12;
+  in.peer_gbs = kModelPeerGBs;  // (host-only plans model a multi-GPU node)
+  in.host_gbs = kModelHostGBs;
+  in.flops_per_s = kModelFlopsPerS;
   if (bound_mode < 0) bound_mode = reuse_bound ? BOUNDS_FIXED : c.opt.bound_model;
   if (bound_mode != BOUNDS_FIXED) in.bound_mode = bound_mode;
   in.window_graphs = choose_window(c, in);
@@ -421,6 +421,10 @@ MICCO_API micco_status micco_plan(micco_ctx *ctx, int32_t n_gpus, const int32_t 
       s.unique_tasks = (int64_t)c.tasks.size();
       s.dedup_hits = c.dedup_hits;
       for (const TaskRec &t : c.tasks) (t.kind == TASK_GEMM ? s.n_gemm : s.n_dot)++;
+      s.model_s = p.predicted_s;
+      for (int64_t b : p.gpu_peak_bytes) s.peak_bytes = std::max(s.peak_bytes, b);
+      s.window_graphs = p.window_graphs;
+      s.model_overlap_s = p.predicted_overlap_s;
       s.n_stages = p.n_stages;
       s.bytes_h2d = p.bytes_h2d;
       s.bytes_p2p = p.bytes_p2p;

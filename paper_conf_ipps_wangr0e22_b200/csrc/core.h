@@ -187,6 +187,7 @@ struct PlanOp {
 
 struct Plan {
   int32_t n_gpus = 1;
+  int32_t window_graphs = 0;
   int32_t reuse_bound[3] = {0, 0, 0};
   std::vector<PlanOp> ops;
   std::vector<int32_t> task_gpu;
@@ -194,6 +195,7 @@ struct Plan {
   int64_t bytes_h2d = 0, bytes_p2p = 0, bytes_d2h = 0, evictions = 0, cache_hits = 0;
   int64_t n_stages = 0;
   double flops = 0, max_over_mean_load = 1, predicted_s = 0;
+  double predicted_overlap_s = 0;  // the same with copies overlapped: Σ_stage max_g max(flops, host, peer)
   std::vector<double> gpu_flops;
   std::vector<std::pair<int32_t, uint64_t>> final_nodes;  // (node tensor, GPU mask) left cached
   std::vector<int32_t> fused_dot;  // GEMM task → DOT task fused into its epilogue, or -1
@@ -246,6 +248,16 @@ struct PlanStream {
     cv.notify_all();
   }
 };
+
+// The planner's cost model (bound sweep, window choice, per-vector labels), calibrated on the
+// B200 (round 2): the TMA GEMM's algorithmic rate on C3 shapes (bench r02: 42.9 TFLOP/s), the
+// pinned H2D copy (55.5 GB/s, profiles/fp64_peak_r01.txt probe), the NVLink peer copy per
+// direction (770 GB/s, B200_PROFILING.md), and a device-local copy between logical GPUs that
+// share one device (half the measured 6550 GB/s copy bandwidth: every byte is read and written).
+constexpr double kModelFlopsPerS = 42.9e12;
+constexpr double kModelHostGBs = 55.5;
+constexpr double kModelPeerGBs = 770.0;
+constexpr double kModelLocalCopyGBs = 3275.0;
 
 struct PlanInput {
   PlanStream *stream = nullptr;                     // optional: publish ops as stages complete

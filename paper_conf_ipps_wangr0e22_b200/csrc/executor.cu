@@ -814,9 +814,9 @@ struct Executor::Impl {
       const char *e = getenv("MICCO_GEMM_TMA");
       use_tma = !(e && e[0] == '0');
     }
-    in.peer_gbs = (ndev > 1 && !dist()) || dist() ? 700 : 2500;
-    in.host_gbs = 55;
-    in.flops_per_s = 30e12;
+    in.peer_gbs = (ndev > 1 && !dist()) || dist() ? kModelPeerGBs : kModelLocalCopyGBs;
+    in.host_gbs = kModelHostGBs;
+    in.flops_per_s = kModelFlopsPerS;
     // node replicas cached by the previous execute: the previous plan's final residency,
     // identical on every rank (the local pointers must agree with it)
     in.initial_nodes.assign(n, {});
@@ -1081,6 +1081,10 @@ struct Executor::Impl {
     st.flops = plan.flops;
     for (const GraphRec &gr : c.graphs) st.flops_no_dedup += gr.flops_no_dedup;
     st.max_over_mean_load = plan.max_over_mean_load;
+    st.model_s = plan.predicted_s;
+    for (int64_t b : plan.gpu_peak_bytes) st.peak_bytes = std::max(st.peak_bytes, b);
+    st.window_graphs = plan.window_graphs;
+    st.model_overlap_s = plan.predicted_overlap_s;
     for (int i = 0; i < 3; ++i) st.reuse_bound[i] = plan.reuse_bound[i];
     st.n_gpus = n;
     if (dist()) {  // plan-level byte counts are global; report them

@@ -161,6 +161,7 @@ Plan make_plan(const Context &ctx, const PlanInput &in) {
 
   // 1. window of every task = window of the first graph that needs it
   const int32_t W = in.window_graphs > 0 ? in.window_graphs : 256;
+  plan.window_graphs = W;
   // Graphs are windowed in an order that keeps graphs sharing an intermediate together:
   // key = the smallest id among the level-1 tasks a graph depends on (its first shared
   // product), ties in graph order.  Shared intermediates then live for a few windows instead
@@ -314,6 +315,7 @@ Plan make_plan(const Context &ctx, const PlanInput &in) {
 
   // One stage (a vector of independent pairs): schedule, simulate the cache, emit the ops,
   // release dead operands.  Returns the stage's modelled time (max over GPUs).
+  double stage_overlap_s = 0;  // the last run_stage's overlapped-copies model
   auto run_stage = [&](int32_t s) -> double {
     S.stage = s;
     sched.begin_vector(stages[s].second - stages[s].first);
@@ -388,12 +390,15 @@ Plan make_plan(const Context &ctx, const PlanInput &in) {
       for (int j = 0; j < k; ++j)
         if (--S.uses_left[ops[j]] == 0) S.release(ops[j]);
     }
-    double worst = 0;
+    double worst = 0, worst_ov = 0;
     for (int g = 0; g < n; ++g) {
-      double tg = S.st_flops[g] / in.flops_per_s + (S.st_h2d[g] + S.st_d2h[g]) / (in.host_gbs * 1e9) +
-                  S.st_p2p[g] / (in.peer_gbs * 1e9);
-      worst = std::max(worst, tg);
+      const double tf = S.st_flops[g] / in.flops_per_s, th = (S.st_h2d[g] + S.st_d2h[g]) / (in.host_gbs * 1e9),
+                   tp = S.st_p2p[g] / (in.peer_gbs * 1e9);
+      worst = std::max(worst, tf + th + tp);
+      // the executor's copy and peer streams overlap the kernels: the optimistic bound
+      worst_ov = std::max(worst_ov, std::max(tf, std::max(th, tp)));
     }
+    stage_overlap_s = worst_ov;
     return worst;
   };
 
@@ -456,7 +461,7 @@ Plan make_plan(const Context &ctx, const PlanInput &in) {
 
   const bool per_stage = in.bound_mode != BOUNDS_FIXED && n > 1 &&
                          (in.policy == MICCO_POLICY_MICCO || in.policy == MICCO_POLICY_MICCO_AFFINITY);
-  double predicted = 0;
+  double predicted = 0, predicted_ov = 0;
   if (in.stream) in.stream->publish_fused(plan.fused_dot);
   for (int32_t s = 0; s < (int32_t)stages.size(); ++s) {
     double f[kBoundFeatures];
@@ -483,6 +488,7 @@ Plan make_plan(const Context &ctx, const PlanInput &in) {
     sched.set_bounds(bd);
     plan.stage_bounds.insert(plan.stage_bounds.end(), bd, bd + 3);
     predicted += run_stage(s);
+    predicted_ov += stage_overlap_s;
     if (in.stream) in.stream->publish_ops(plan.ops);  // this stage's ops are final
   }
   if (in.keep_inputs)
@@ -490,6 +496,7 @@ Plan make_plan(const Context &ctx, const PlanInput &in) {
       if (S.mask[x] && ctx.tensors[x].node >= 0) plan.final_nodes.push_back({x, S.mask[x]});
   plan.n_stages = (int64_t)stages.size();
   plan.predicted_s = predicted;
+  plan.predicted_overlap_s = predicted_ov;
   double mx = 0, sum = 0;
   for (double f : plan.gpu_flops) { mx = std::max(mx, f); sum += f; }
   plan.max_over_mean_load = sum > 0 ? mx / (sum / n) : 1.0;

@@ -58,7 +58,9 @@ class micco_stats(ctypes.Structure):
                 ("enqueue_ms", ctypes.c_double), ("host_pinned", ctypes.c_int32), ("gemm_3m", ctypes.c_int32),
                 ("gemm_dmma_flops", ctypes.c_double), ("dot_main_ms", ctypes.c_double),
                 ("dot_main_bytes", ctypes.c_double), ("dot_main_launches", ctypes.c_int64),
-                ("plan_ms", ctypes.c_double), ("gemm_tma_launches", ctypes.c_int64)]
+                ("plan_ms", ctypes.c_double), ("gemm_tma_launches", ctypes.c_int64),
+                ("model_s", ctypes.c_double), ("model_overlap_s", ctypes.c_double),
+                ("peak_bytes", ctypes.c_int64), ("window_graphs", ctypes.c_int32)]
 
     def as_dict(self) -> Dict:
         d = {}

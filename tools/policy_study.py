@@ -11,7 +11,7 @@ Uniform / Gaussian node selection, at 2 / 4 / 8 GPUs, every policy is planned on
   least_loaded  Groute's rule: the GPU with the least assigned work
 
 and reports per plan: the modelled time (planner cost model: per stage, max over GPUs of
-flops / 30 TF/s + host bytes / 55 GB/s + peer bytes / 700 GB/s), H2D and P2P bytes, cache
+flops / 42.9 TF/s + host bytes / 55.5 GB/s + peer bytes / 770 GB/s), H2D and P2P bytes, cache
 hits, evictions, max/mean load and the host planning time (host_s).  The modelled time is a model,
 not a measurement (the GPU box has one B200); bytes, hits and load balance are exact
 properties of the plans the executor replays.
@@ -76,7 +76,7 @@ def main(argv=None):
                                  for x in rows[-len(POLICIES):])
                 print(f"{dist:8s} r={r:.1f} n={n}: {line}", flush=True)
     meta = {"graphs": a.graphs, "N": a.N, "Lt": a.Lt, "window_graphs": a.window, "budget_gb": a.budget_gb,
-            "cost_model": "per stage max over GPUs of flops/30 TF/s + host bytes/55 GB/s + peer bytes/700 GB/s",
+            "cost_model": "per stage max over GPUs of flops/42.9 TF/s + host bytes/55.5 GB/s + peer bytes/770 GB/s",
             "note": "modelled plan time (host-only planning); bytes, hits and load are exact plan properties"}
     Path(a.out).write_text(json.dumps({"meta": meta, "rows": rows}, indent=1))
     print("wrote", a.out)
