@@ -201,7 +201,7 @@ struct Executor::Impl {
   size_t vals_elems = 0;
   int vals_dev = 0;
   double2 *h_corr = nullptr;
-  int64_t launches = 0, tma_launches = 0;
+  int64_t launches = 0, tma_launches = 0, oom_retries = 0;
   bool use_tma = true;  // TMA GEMM for the contractions that fit it (see execute)
   bool dist() const { return c.opt.dist_world > 0; }
   int table_of(int i) const { return c.opt.scalar_tables ? i : g[i].dev; }
@@ -411,10 +411,43 @@ struct Executor::Impl {
     if (nf >= 2) CK(cudaStreamWaitEvent(l.pst, l.flush_ev[nf - 2], 0));
   }
 
-  double2 *alloc(LGpu &l, int64_t bytes) {
+  double2 *alloc(LGpu &l, int64_t bytes) { return (double2 *)alloc_on(l, bytes, l.st); }
+
+  // A stream-ordered allocation that survives transient pool pressure.  The plan keeps each
+  // GPU's live set inside its budget in plan order, but the copy and peer streams run ahead of
+  // the compute stream, so an allocation can be made while frees the plan placed before it are
+  // still queued behind kernels, and the pool cannot hand their blocks out yet; with very large
+  // tensors (C5's 17.2 GB rank-4 intermediates) and a budget near the device size that can
+  // exhaust the device.  On an out-of-memory error: drain this device's streams (the queued
+  // frees complete), retry; then return the pool's cached blocks to the driver, retry; only then
+  // fail (MICCO_ERR_OOM).
+  void *alloc_on(LGpu &l, int64_t bytes, cudaStream_t s) {
     void *p = nullptr;
-    CK(cudaMallocAsync(&p, (size_t)bytes, l.st));
-    return (double2 *)p;
+    cudaError_t e = cudaMallocAsync(&p, (size_t)bytes, s);
+    if (e == cudaErrorMemoryAllocation) {
+      cudaGetLastError();  // (not sticky)
+      for (auto &o : g)
+        if (o.local && o.dev == l.dev) {
+          CK(cudaStreamSynchronize(o.st));
+          CK(cudaStreamSynchronize(o.cst));
+          CK(cudaStreamSynchronize(o.pst));
+        }
+      ++oom_retries;
+      e = cudaMallocAsync(&p, (size_t)bytes, s);
+      if (e == cudaErrorMemoryAllocation) {
+        cudaGetLastError();
+        cudaMemPool_t pool;
+        CK(cudaDeviceGetDefaultMemPool(&pool, l.dev));
+        CK(cudaMemPoolTrimTo(pool, 0));
+        e = cudaMallocAsync(&p, (size_t)bytes, s);
+      }
+      if (e == cudaErrorMemoryAllocation) {
+        cudaGetLastError();
+        fail(MICCO_ERR_OOM, "device allocation of " + std::to_string(bytes) + " B failed after draining the streams");
+      }
+    }
+    CK(e);
+    return p;
   }
 
   int64_t bytes_of(int32_t x) const { return c.tensors[x].bytes(c.Lt); }
@@ -644,7 +677,7 @@ struct Executor::Impl {
         auto it = spill_ev.find(op.id);  // a spilled intermediate: wait for its D2H
         if (it != spill_ev.end() && c.tensors[op.id].node < 0) CK(cudaStreamWaitEvent(l.cst, it->second.second, 0));
         void *p = nullptr;
-        CK(cudaMallocAsync(&p, (size_t)bytes_of(op.id), l.cst));
+        p = alloc_on(l, bytes_of(op.id), l.cst);
         Timed tm{devs[l.dev].timing_events.get(), devs[l.dev].timing_events.get(), 2, l.dev};
         CK(cudaEventRecord(tm.a, l.cst));
         CK(cudaMemcpyAsync(p, host_src(op.id), bytes_of(op.id), cudaMemcpyHostToDevice, l.cst));
@@ -666,8 +699,7 @@ struct Executor::Impl {
             CK(cudaSetDevice(dst.dev));
             cudaStream_t s = dst.pst;
             pace_peer(dst);
-            void *p = nullptr;
-            CK(cudaMallocAsync(&p, (size_t)nb, s));
+            void *p = alloc_on(dst, nb, s);
             NK(nccl().Recv(p, (size_t)nb / 8, ncclDouble, op.src, comm, s));
             CK(cudaStreamWaitEvent(dst.st, record_on(op.gpu, s), 0));  // consumers wait
             dst.ptr[op.id] = (double2 *)p;
@@ -685,9 +717,7 @@ struct Executor::Impl {
         cudaStream_t s = dst.pst;
         CK(cudaStreamWaitEvent(s, ready, 0));
         pace_peer(dst);
-        void *pv = nullptr;
-        CK(cudaMallocAsync(&pv, (size_t)nb, s));
-        double2 *p = (double2 *)pv;
+        double2 *p = (double2 *)alloc_on(dst, nb, s);
         if (dst.dev == src.dev)
           CK(cudaMemcpyAsync(p, src.ptr[op.id], nb, cudaMemcpyDeviceToDevice, s));
         else
@@ -793,6 +823,7 @@ struct Executor::Impl {
       if (l.local && l.ptr.size() < c.tensors.size()) l.ptr.resize(c.tensors.size(), nullptr);
     launches = 0;
     tma_launches = 0;
+    oom_retries = 0;
     timed.clear();
     for (auto &l : g) {
       l.flush_ev.clear();
@@ -1078,6 +1109,7 @@ struct Executor::Impl {
     st.n_stages = plan.n_stages;
     st.kernel_launches = launches;
     st.gemm_tma_launches = tma_launches;
+    st.alloc_retries = oom_retries;
     st.flops = plan.flops;
     for (const GraphRec &gr : c.graphs) st.flops_no_dedup += gr.flops_no_dedup;
     st.max_over_mean_load = plan.max_over_mean_load;

@@ -60,7 +60,8 @@ class micco_stats(ctypes.Structure):
                 ("dot_main_bytes", ctypes.c_double), ("dot_main_launches", ctypes.c_int64),
                 ("plan_ms", ctypes.c_double), ("gemm_tma_launches", ctypes.c_int64),
                 ("model_s", ctypes.c_double), ("model_overlap_s", ctypes.c_double),
-                ("peak_bytes", ctypes.c_int64), ("window_graphs", ctypes.c_int32)]
+                ("peak_bytes", ctypes.c_int64), ("window_graphs", ctypes.c_int32),
+                ("alloc_retries", ctypes.c_int64)]
 
     def as_dict(self) -> Dict:
         d = {}

@@ -64,6 +64,7 @@ def run(wl, budget, window, warm_steps=2):
                "evictions": st["evictions"], "bytes_h2d": st["bytes_h2d"], "bytes_d2h": st["bytes_d2h"],
                "bytes_p2p": st["bytes_p2p"], "cold_bytes_h2d": cst["bytes_h2d"], "cold_bytes_d2h": cst["bytes_d2h"],
                "peak_gb": st["peak_bytes"] / 1e9, "gemm_ms": st["gemm_kernel_ms"], "copy_ms": st["copy_ms"],
+               "alloc_retries": st["alloc_retries"] + cst["alloc_retries"],
                "tflops": st["flops"] / (np.mean(ms) / 1e3) / 1e12}
 
 
@@ -79,6 +80,7 @@ def main(argv=None):
     ap = argparse.ArgumentParser()
     ap.add_argument("--out", default=str(ROOT / "gpurun_out" / "c5_sweep_r02.json"))
     ap.add_argument("--skip-full", action="store_true")
+    ap.add_argument("--skip-small", action="store_true")
     a = ap.parse_args(argv)
     out = {"rows": []}
     wl = workloads.c5_mixed(n_combos=1, Nb=64, Nm=256, Lt=16, pool=2, meson_graphs=64)
@@ -86,7 +88,7 @@ def main(argv=None):
     out["c5_demand_gb"] = d / 1e9
     print(f"c5: {len(wl.graphs)} graphs, demand at W=256: {d / 1e9:.1f} GB", flush=True)
     ref = None
-    for pct in (125, 150, 175, 200):
+    for pct in ([] if a.skip_small else (125, 150, 175, 200)):
         for window in (256, 0):
             t0 = time.perf_counter()
             C, r = run(wl, d * 100 / pct, window)
