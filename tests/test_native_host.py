@@ -306,3 +306,48 @@ def test_affinity_policy_cuts_peer_traffic():
     assert res["micco_affinity"]["bytes_p2p"] < 0.7 * res["micco"]["bytes_p2p"]
     assert res["micco_affinity"]["max_over_mean_load"] < 1.1
     assert res["micco_affinity"]["n_gemm"] == res["micco"]["n_gemm"]
+
+
+def test_plan_model_and_demand_stats():
+    """micco_plan reports the plan's window, its peak resident bytes (the memory demand C5's
+    oversubscription sweep sets budgets from) and both cost-model times: copies overlapped
+    (Σ_stage max_g max(flops, host, peer)) never exceeds copies serialised."""
+    wl = workloads.c2_meson_set(n_graphs=200, N=16, Lt=4, rate=0.6, dist="gaussian")
+    node = 16 * 16 * 4 * 16
+    big = _ctx(mem_budget_bytes=1 << 40, window_graphs=32)
+    M.load_workload(big, wl)
+    st, _ = big.plan(2, [1, 1, 0])
+    assert st["window_graphs"] == 32
+    assert 0 < st["model_overlap_s"] <= st["model_s"]
+    assert st["peak_bytes"] >= node and st["evictions"] == 0
+    demand = st["peak_bytes"]
+    tight = _ctx(mem_budget_bytes=demand // 2, window_graphs=32)
+    M.load_workload(tight, wl)
+    st2, _ = tight.plan(2, [1, 1, 0])
+    assert st2["peak_bytes"] <= demand // 2 and st2["evictions"] > 0
+    auto = _ctx(mem_budget_bytes=demand // 2)  # window_graphs = 0: sized to the budget
+    M.load_workload(auto, wl)
+    st3, _ = auto.plan(2, [1, 1, 0])
+    assert st3["window_graphs"] >= 1 and st3["peak_bytes"] <= demand // 2
+
+
+def test_set_policy_and_scalar_tables_options():
+    ctx = _ctx()
+    M.micco_set_policy(ctx.h, "round_robin")
+    with pytest.raises(M.MiccoError):
+        M.micco_set_policy(ctx.h, 9)
+    M.Context(scalar_tables=1, mem_budget_bytes=1 << 30).close()
+    with pytest.raises(M.MiccoError):
+        M.Context(scalar_tables=2)
+
+
+def test_graph_beyond_kernel_limits_rejected_at_add_graph():
+    """A contraction whose slice exceeds the kernels' 32-bit per-slice offsets is refused when
+    the graph is added (MICCO_ERR_UNSUPPORTED), not part-way through an execute: the full dot
+    of two N = 1300 baryons reads slices of 1300^3 = 2.2e9 > 2^31 elements (synthetic nodes are
+    generated lazily, so nothing is allocated)."""
+    ctx = _ctx()
+    ids = ctx.add_nodes_synth(3, 1300, 1, 1, [1, 2], 0, 1.0)
+    with pytest.raises(M.MiccoError) as e:
+        ctx.add_graph([int(ids[0]), int(ids[1])], [(0, 0, 1, 0), (0, 1, 1, 1), (0, 2, 1, 2)], [0, 1, 2])
+    assert e.value.status == -4
