@@ -343,11 +343,16 @@ def test_set_policy_and_scalar_tables_options():
 
 def test_graph_beyond_kernel_limits_rejected_at_add_graph():
     """A contraction whose slice exceeds the kernels' 32-bit per-slice offsets is refused when
-    the graph is added (MICCO_ERR_UNSUPPORTED), not part-way through an execute: the full dot
-    of two N = 1300 baryons reads slices of 1300^3 = 2.2e9 > 2^31 elements (synthetic nodes are
-    generated lazily, so nothing is allocated)."""
+    the graph is added (MICCO_ERR_UNSUPPORTED), not part-way through an execute: two N = 216
+    baryons joined by one leg first (the other legs run through two mesons) give a rank-4
+    intermediate with 216^4 = 2.18e9 > 2^31 elements per slice."""
     ctx = _ctx()
-    ids = ctx.add_nodes_synth(3, 1300, 1, 1, [1, 2], 0, 1.0)
+    N = 216
+    bar = ctx.add_nodes_synth(3, N, 1, 1, [1, 2], 0, 1.0)
+    mes = ctx.add_nodes_synth(2, N, 1, 1, [3, 4], 0, 1.0)
+    inst = [int(bar[0]), int(bar[1]), int(mes[0]), int(mes[1])]
+    edges = [(0, 0, 1, 0), (0, 1, 2, 0), (0, 2, 3, 0), (1, 1, 2, 1), (1, 2, 3, 1)]
     with pytest.raises(M.MiccoError) as e:
-        ctx.add_graph([int(ids[0]), int(ids[1])], [(0, 0, 1, 0), (0, 1, 1, 1), (0, 2, 1, 2)], [0, 1, 2])
+        ctx.add_graph(inst, edges, [0, 1, 2, 3, 4])
     assert e.value.status == -4
+    ctx.close()
