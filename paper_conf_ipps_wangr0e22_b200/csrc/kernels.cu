@@ -1382,6 +1382,11 @@ bool gemm_tma_class(const GemmDesc &d, int *cls) {
   if (ak ? (d.Ko > 1 && d.Mo > 1) : (d.Ko > 1 || d.Mo > 1 || d.Mi % 2 != 0)) return false;
   if (bk ? (d.Ko > 1 && d.No > 1) : (d.Ko > 1 || d.No > 1 || d.Ni % 2 != 0)) return false;
   if ((((uintptr_t)d.A) | ((uintptr_t)d.B)) & 15) return false;
+  // The TMA kernel's tile is 128 rows: a short M (C4/C5's single N = 64 leg, C1's N = 32)
+  // would leave most of it zero-filled; the 64-row cp.async kernel takes those (C5 at its
+  // stated size: 8.4 s per step on the 128-row tile against 6.9 s).
+  const int tm = (d.Mi + TM_BM - 1) / TM_BM * TM_BM;
+  if (8 * tm > 9 * d.Mi) return false;  // more than 1/9 of the tile's rows wasted
   *cls = kGemmClassTMA + (ak ? 0 : 2) + (bk ? 1 : 0);
   return true;
 }

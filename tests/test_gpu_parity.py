@@ -414,8 +414,8 @@ def test_gemm_paths_meson_shapes(tma, monkeypatch):
     with the reuse-aware order (fused final dots), ≤ 1e-10 against the oracle, and integer
     inputs bit-exact; the TMA run must really use the TMA kernel."""
     monkeypatch.setenv("MICCO_GEMM_TMA", tma)
-    for wl in (workloads.c2_meson_set(n_graphs=60, N=64, Lt=3, rate=0.5, flips=True),
-               workloads.c3_multi_meson(n_graphs=40, N=96, Lt=2, pool=4)):
+    for wl in (workloads.c2_meson_set(n_graphs=60, N=128, Lt=3, rate=0.5, flips=True),
+               workloads.c3_multi_meson(n_graphs=40, N=128, Lt=2, pool=4)):
         C, st = check(wl, reorder=True)
         assert (st["gemm_tma_launches"] > 0) == (tma == "1"), st
         assert st["gemm_tma_launches"] <= st["gemm_launches"]
@@ -423,3 +423,22 @@ def test_gemm_paths_meson_shapes(tma, monkeypatch):
     _, vals, _ = run_gpu(wli)
     _, valso = oracle.correlator(wli, return_values=True)
     assert np.array_equal(vals, valso)
+
+
+def test_tma_gemm_ragged_tiles():
+    """The TMA kernel's zero-filled boxes: meson cycles at N = 1032 (the smallest N above 1024
+    whose 128-row tiles it takes: 1032 = 8·128 + 8 rows, 32·32 + 8 columns, k = 64·16 + 8), so
+    every tile edge and the last k-stage are ragged; all four operand-layout classes via random
+    transposes; ≤ 1e-10 against the oracle and the TMA kernel really used."""
+    rng = np.random.default_rng(5)
+    N = 1032
+    nodes = [NodeSpec(2, N, 700 + i) for i in range(3)]
+    graphs = []
+    for k in (2, 3, 3, 2):
+        inst = [int(x) for x in rng.integers(0, 3, size=k)]
+        flips = [bool(x) for x in rng.integers(0, 2, size=k)]
+        graphs.append(GraphSpec(inst, workloads.meson_cycle_edges(k, flips), list(range(k)),
+                                complex(rng.choice([-1.0, 1.0]))))
+    wl = Workload("ragged1032", 1, 91, 0, nodes, graphs)
+    C, st = check(wl)
+    assert st["gemm_tma_launches"] > 0, st
