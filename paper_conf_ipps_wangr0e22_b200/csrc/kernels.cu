@@ -877,7 +877,12 @@ __device__ __forceinline__ void zgemm_tma_body(const GemmTmaBatch &b, long long 
       if (kq + 1 < TM_BK / 4) {
         load_frag(cur ^ 1, slot, kq + 1);
       } else {
-        // every fragment of this slot is in registers (and summed): hand the slot back
+        // Every fragment of this slot has been read: hand the slot back.  The reads are generic-
+        // proxy LDS and the next write to the slot is the producer's TMA (async proxy): without
+        // a proxy fence the arrive could overtake LDS still queued (ptxas schedules the last
+        // k-quad's LDS a few instructions before it), and a fast TMA overwrote the slot under
+        // them about once per 20 C3 executes (one wrong fused-dot partial; tools/race_hunt.py).
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
         __syncwarp();
         if (lane == 0) mbar_arrive(empty0 + 8 * slot);
         if (++slot == TM_ST) { slot = 0; ph ^= 1; }

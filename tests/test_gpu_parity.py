@@ -442,3 +442,27 @@ def test_tma_gemm_ragged_tiles():
     wl = Workload("ragged1032", 1, 91, 0, nodes, graphs)
     C, st = check(wl)
     assert st["gemm_tma_launches"] > 0, st
+
+
+def test_repeat_bitwise_at_scale():
+    """Bitwise reproducibility of every graph value over repeated executes and fresh contexts at
+    C3's tensor size (N = 256, Lt = 128, 2000 graphs, reuse-aware order: TMA GEMMs with fused
+    dots).  Guards the TMA ring's slot release: without the proxy fence before the consumers'
+    empty-barrier arrive, a TMA write could overtake queued LDS of the slot it refills (about one
+    wrong (graph, slice) per 20 executes of 10k graphs; tools/race_hunt.py)."""
+    wl = workloads.c3_multi_meson(n_graphs=2000, N=256, Lt=128)
+    ref = None
+    for _ in range(2):
+        ctx = M.Context(keep_inputs_resident=True, reorder=True)
+        M.load_workload(ctx, wl)
+        for _ in range(3):
+            ctx.execute(1)
+            st = ctx.stats()
+            assert st["gemm_tma_launches"] > 0
+            vals = np.array([[ctx.graph_value(g, t) for t in range(wl.Lt)] for g in range(len(wl.graphs))])
+            if ref is None:
+                ref = vals
+            else:
+                bad = np.argwhere(vals != ref)
+                assert len(bad) == 0, bad[:10]
+        ctx.close()

@@ -108,6 +108,7 @@ __global__ void stream_kernel(const __grid_constant__ Maps m, int iters, int R, 
     const int slot = it & 3;
     mbar_wait(&bar[slot], (it >> 2) & 1);
     acc += ring[slot * 1024 + threadIdx.x].x;
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // generic reads before the next TMA write
     __syncthreads();  // the slot is free again
     if (threadIdx.x == 0 && it + 4 < iters) issue(it + 4);
   }
