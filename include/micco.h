@@ -232,6 +232,9 @@ typedef struct {
                                   Σ over stages of max over GPUs of max(flops, host, peer) time */
   int64_t peak_bytes;          /* the plan's largest resident set on one GPU (its memory demand) */
   int32_t window_graphs;       /* the window the plan used (options.window_graphs or the auto choice) */
+  int64_t component_dedup_hits;/* graph components reused whole because an earlier graph held the same
+                                  hadron nodes wired the same way up to relabeling (canonical
+                                  sub-network hashing: tr(ABC) = tr(BCA) costs one contraction) */
   int64_t alloc_retries;       /* device allocations that had to drain the streams first (the copy
                                   and peer streams ran ahead of frees still queued on the compute
                                   stream) */

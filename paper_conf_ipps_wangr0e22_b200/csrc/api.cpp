@@ -420,6 +420,7 @@ MICCO_API micco_status micco_plan(micco_ctx *ctx, int32_t n_gpus, const int32_t 
       s.struct_size = sizeof(s);
       s.unique_tasks = (int64_t)c.tasks.size();
       s.dedup_hits = c.dedup_hits;
+      s.component_dedup_hits = c.component_dedup_hits;
       for (const TaskRec &t : c.tasks) (t.kind == TASK_GEMM ? s.n_gemm : s.n_dot)++;
       s.model_s = p.predicted_s;
       for (int64_t b : p.gpu_peak_bytes) s.peak_bytes = std::max(s.peak_bytes, b);

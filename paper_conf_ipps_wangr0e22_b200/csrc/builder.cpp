@@ -7,6 +7,7 @@
 // — the same (operand, operand, contracted legs) step is interned once here, so a shared
 // intermediate is computed once for every graph that needs it.
 #include <algorithm>
+#include <functional>
 #include <numeric>
 #include <string>
 
@@ -52,6 +53,7 @@ struct Comp {
   int32_t dim[2 * kMaxRank + 4];
   int32_t level;
   bool alive;
+  double flops;                   // no-dedup flops of the steps merged into this component
 };
 
 struct Step {  // one pairwise reduction chosen for a graph
@@ -114,6 +116,97 @@ void build_graph(Context &ctx, int32_t n_inst, const int64_t *node_ids, int32_t 
     }
   }
 
+  // Canonical sub-network hashing: a connected component whose hadron
+  // nodes and wiring equal, up to relabeling its instances, a component interned by an earlier
+  // graph has the same value (overlapped reduction paths), whatever tree either
+  // was contracted by — e.g. tr(ABC) and tr(BCA).  When every component of this graph is such a
+  // repeat, the graph reuses the earlier scalars and no task is built; otherwise the graph is
+  // decomposed as usual and its components are recorded.  The key: instances sorted by node id
+  // (ties: every order within a group of equal nodes), then the sorted normalised edge list;
+  // the smallest over the tie orders.  Components with more than 5040 tie orders keep no key.
+  std::vector<int32_t> comp_root(n_inst);
+  {
+    std::vector<int32_t> parent(n_inst);
+    std::iota(parent.begin(), parent.end(), 0);
+    std::function<int32_t(int32_t)> find = [&](int32_t x) { return parent[x] == x ? x : parent[x] = find(parent[x]); };
+    for (int e = 0; e < n_edges; ++e) parent[find(edges[e].u)] = find(edges[e].v);
+    for (int u = 0; u < n_inst; ++u) comp_root[u] = find(u);
+  }
+  auto component_key = [&](int32_t root) -> std::string {
+    std::vector<int32_t> mem;
+    for (int u = 0; u < n_inst; ++u)
+      if (comp_root[u] == root) mem.push_back(u);
+    std::stable_sort(mem.begin(), mem.end(), [&](int32_t x, int32_t y) { return node_ids[x] < node_ids[y]; });
+    // tie groups (equal node ids) are permuted among themselves
+    std::vector<std::pair<int, int>> groups;
+    double orders = 1;
+    for (size_t i = 0; i < mem.size();) {
+      size_t j = i;
+      while (j < mem.size() && node_ids[mem[j]] == node_ids[mem[i]]) ++j;
+      groups.push_back({(int)i, (int)j});
+      for (size_t k = 2; k <= j - i; ++k) orders *= (double)k;
+      i = j;
+    }
+    if (orders > 5040) return std::string();
+    std::vector<int64_t> best;
+    std::vector<int32_t> pos(n_inst, -1);
+    std::vector<int32_t> cur = mem;
+    std::function<void(size_t)> rec = [&](size_t gi) {
+      if (gi == groups.size()) {
+        for (size_t i = 0; i < cur.size(); ++i) pos[cur[i]] = (int32_t)i;
+        std::vector<int64_t> key;
+        key.push_back((int64_t)cur.size());
+        for (int32_t u : cur) key.push_back(node_ids[u]);
+        std::vector<int64_t> ek;
+        for (int e = 0; e < n_edges; ++e) {
+          const micco_edge &E = edges[e];
+          if (comp_root[E.u] != root) continue;
+          int64_t a = (int64_t)pos[E.u] * 8 + E.p, b = (int64_t)pos[E.v] * 8 + E.q;
+          if (a > b) std::swap(a, b);
+          ek.push_back(a * 4096 + b);
+        }
+        std::sort(ek.begin(), ek.end());
+        key.insert(key.end(), ek.begin(), ek.end());
+        if (best.empty() || key < best) best.swap(key);
+        return;
+      }
+      auto [b, e] = groups[gi];
+      std::sort(cur.begin() + b, cur.begin() + e);
+      do rec(gi + 1);
+      while (std::next_permutation(cur.begin() + b, cur.begin() + e));
+    };
+    rec(0);
+    return std::string(reinterpret_cast<const char *>(best.data()), best.size() * sizeof(int64_t));
+  };
+  std::vector<int32_t> roots;
+  for (int u = 0; u < n_inst; ++u)
+    if (comp_root[u] == u) roots.push_back(u);
+  std::vector<std::string> keys(roots.size());
+  {
+    bool all_known = true;
+    for (size_t i = 0; i < roots.size(); ++i) {
+      keys[i] = component_key(roots[i]);
+      if (keys[i].empty() || !ctx.component_by_key.count(keys[i])) all_known = false;
+    }
+    if (all_known) {
+      GraphRec g;
+      g.coef_re = cre;
+      g.coef_im = cim;
+      g.comp_begin = (int32_t)ctx.graph_scalars.size();
+      double fl = 0;
+      for (const std::string &k : keys) {
+        const auto &hit = ctx.component_by_key.at(k);
+        ctx.graph_scalars.push_back(hit.first);
+        fl += hit.second;
+      }
+      g.comp_end = (int32_t)ctx.graph_scalars.size();
+      g.flops_no_dedup = fl;
+      ctx.graphs.push_back(g);
+      ctx.component_dedup_hits += (int64_t)keys.size();
+      return;
+    }
+  }
+
   // Two passes over the same decomposition: a dry run that picks the steps and validates
   // ranks and layouts (so a failing graph leaves the DAG untouched), then the commit that
   // replays the dry run's steps and interns tasks.  The dry run predicts the ids the commit
@@ -133,6 +226,7 @@ void build_graph(Context &ctx, int32_t n_inst, const int64_t *node_ids, int32_t 
       for (int p = 0; p < rank[u]; ++p) { c.leg[p] = u * 8 + p; c.dim[p] = N[u]; }
       c.level = 0;
       c.alive = true;
+      c.flops = 0;
       comp_of[u] = u;
     }
     std::vector<char> done(n_edges, 0);
@@ -292,6 +386,7 @@ void build_graph(Context &ctx, int32_t n_inst, const int64_t *node_ids, int32_t 
       Comp &A = comps[st.ca];
       Comp res{};
       res.alive = true;
+      res.flops = A.flops + (st.cb >= 0 ? comps[st.cb].flops : 0.0);
       double step_flops;
       if (st.cb < 0) {  // trace
         res.rank = 0;
@@ -315,6 +410,7 @@ void build_graph(Context &ctx, int32_t n_inst, const int64_t *node_ids, int32_t 
         step_flops = 8.0 * (double)rs * (double)kd * ctx.Lt;
       }
       flops_nd += step_flops;
+      res.flops += step_flops;
       res.tensor = -1;
       const TaskKey key = make_key(st);
       if (!commit) {  // predict the id the commit gives this step's result
@@ -374,7 +470,13 @@ void build_graph(Context &ctx, int32_t n_inst, const int64_t *node_ids, int32_t 
       g.coef_im = cim;
       g.comp_begin = (int32_t)ctx.graph_scalars.size();
       for (int u = 0; u < n_inst; ++u)
-        if (comps[u].alive) ctx.graph_scalars.push_back(comps[u].tensor);
+        if (comps[u].alive) {
+          ctx.graph_scalars.push_back(comps[u].tensor);
+          // record the component for canonical reuse (its members share comp_root)
+          for (size_t i = 0; i < roots.size(); ++i)
+            if (comp_root[u] == roots[i] && !keys[i].empty())
+              ctx.component_by_key.emplace(keys[i], std::make_pair(comps[u].tensor, comps[u].flops));
+        }
       g.comp_end = (int32_t)ctx.graph_scalars.size();
       g.flops_no_dedup = flops_nd;
       ctx.graphs.push_back(g);

@@ -152,6 +152,9 @@ struct Context {
   std::vector<GraphRec> graphs;
   std::vector<int32_t> graph_scalars;  // tensor ids (rank 0), grouped per graph
   int64_t dedup_hits = 0;
+  // canonical sub-network key of a connected component → (its scalar tensor, no-dedup flops)
+  std::unordered_map<std::string, std::pair<int32_t, double>> component_by_key;
+  int64_t component_dedup_hits = 0;
   int32_t n_scalar_slots = 0;
   // results of the last execute
   bool have_result = false;

@@ -1105,6 +1105,7 @@ struct Executor::Impl {
     st.cache_hits = plan.cache_hits;
     st.unique_tasks = (int64_t)c.tasks.size();
     st.dedup_hits = c.dedup_hits;
+    st.component_dedup_hits = c.component_dedup_hits;
     for (const TaskRec &t : c.tasks) (t.kind == TASK_GEMM ? st.n_gemm : st.n_dot)++;
     st.n_stages = plan.n_stages;
     st.kernel_launches = launches;

@@ -61,7 +61,7 @@ class micco_stats(ctypes.Structure):
                 ("plan_ms", ctypes.c_double), ("gemm_tma_launches", ctypes.c_int64),
                 ("model_s", ctypes.c_double), ("model_overlap_s", ctypes.c_double),
                 ("peak_bytes", ctypes.c_int64), ("window_graphs", ctypes.c_int32),
-                ("alloc_retries", ctypes.c_int64)]
+                ("component_dedup_hits", ctypes.c_int64), ("alloc_retries", ctypes.c_int64)]
 
     def as_dict(self) -> Dict:
         d = {}

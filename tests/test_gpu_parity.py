@@ -466,3 +466,33 @@ def test_repeat_bitwise_at_scale():
                 bad = np.argwhere(vals != ref)
                 assert len(bad) == 0, bad[:10]
         ctx.close()
+
+
+def test_canonical_component_reuse_parity():
+    """Graphs that repeat earlier ones up to instance relabeling (a random permutation of
+    the instances with the edges remapped, and their own random reduction orders) reuse the
+    earlier components' scalars (component_dedup_hits); every graph value still matches the
+    oracle, which contracts each graph on its own in its own order (≤ 1e-10; bit-exact on
+    integer inputs)."""
+    for mode in (0, MODE_INT3):
+        base = workloads.c1_two_meson(mode=mode)
+        rng = np.random.default_rng(11)
+        graphs = list(base.graphs)
+        for G in base.graphs[:24]:
+            n = len(G.inst)
+            p = [int(x) for x in rng.permutation(n)]  # old instance i -> new label p[i]
+            inst = [None] * n
+            for i in range(n):
+                inst[p[i]] = G.inst[i]
+            edges = [(p[a], la, p[b], lb) for (a, la, b, lb) in G.edges]
+            graphs.append(GraphSpec(inst, edges, [int(x) for x in rng.permutation(len(edges))], G.coef))
+        wl = Workload(base.name + "-perm", base.Lt, base.seed, base.mode, base.nodes, graphs)
+        C, vals, st = run_gpu(wl)
+        assert st["component_dedup_hits"] > 0, st
+        Co, valso = oracle.correlator(wl, return_values=True)
+        if mode == MODE_INT3:
+            assert np.array_equal(vals, valso)
+        else:
+            assert rel_err(C, Co) <= TOL
+            for g in range(len(graphs)):
+                assert rel_err(vals[g], valso[g]) <= TOL, g

@@ -97,10 +97,10 @@ def test_hash_consing_counts():
     # tasks: dot(A,B), gemm(A,B), dot(AB,C), dot(AB,D)
     assert st["unique_tasks"] == 4 and st["n_gemm"] == 1 and st["n_dot"] == 3
     assert st["dedup_hits"] == 1
-    # identical graph again: everything is a hit
+    # identical graph again: its one component is reused whole (canonical sub-network hashing)
     ctx.add_graph([A, B, C], workloads.meson_cycle_edges(3), [0, 1, 2])
     st2, _ = ctx.plan(1, [0, 0, 0])
-    assert st2["unique_tasks"] == 4 and st2["dedup_hits"] == 3
+    assert st2["unique_tasks"] == 4 and st2["component_dedup_hits"] == 1 and st2["dedup_hits"] == 1
 
 
 def test_flops_accounting():
@@ -242,9 +242,9 @@ def test_reorder_dry_run_leaves_dag_untouched_on_failure():
         ctx.add_graph(ids, [(0, 1, 1, 0), (1, 1, 2, 0), (2, 1, 2, 0)], None)  # leg (2, 0) twice
     st1, _ = ctx.plan(1, [0, 0, 0])
     assert st1["unique_tasks"] == st0["unique_tasks"]
-    ctx.add_graph([ids[1], ids[2], ids[0]], workloads.meson_cycle_edges(3), None)  # rotation: all hits
+    ctx.add_graph([ids[1], ids[2], ids[0]], workloads.meson_cycle_edges(3), None)  # rotation: reused whole
     st2, _ = ctx.plan(1, [0, 0, 0])
-    assert st2["unique_tasks"] == st0["unique_tasks"] and st2["dedup_hits"] == st0["dedup_hits"] + 2
+    assert st2["unique_tasks"] == st0["unique_tasks"] and st2["component_dedup_hits"] == 1
 
 
 def test_policy_study_modelled_time(tmp_path):
@@ -303,7 +303,9 @@ def test_affinity_policy_cuts_peer_traffic():
         M.load_workload(ctx, wl)
         res[pol], _ = ctx.plan(4, [1, 1, 1])
         ctx.close()
-    assert res["micco_affinity"]["bytes_p2p"] < 0.7 * res["micco"]["bytes_p2p"]
+    # (0.75: repeated cycles of these r = 0.9 sets are now reused whole by canonical
+    # sub-network hashing, which changes the task mix; the ratio is 0.72 with it)
+    assert res["micco_affinity"]["bytes_p2p"] < 0.75 * res["micco"]["bytes_p2p"]
     assert res["micco_affinity"]["max_over_mean_load"] < 1.1
     assert res["micco_affinity"]["n_gemm"] == res["micco"]["n_gemm"]
 
@@ -356,3 +358,35 @@ def test_graph_beyond_kernel_limits_rejected_at_add_graph():
         ctx.add_graph(inst, edges, [0, 1, 2, 3, 4])
     assert e.value.status == -4
     ctx.close()
+
+
+def test_canonical_component_reuse():
+    """Canonical sub-network hashing: a connected component equal to an
+    earlier one up to relabeling its instances is reused whole — cyclic rotations of a meson
+    trace and reordered disconnected components; a graph with one new component is decomposed
+    as usual (its known component's steps are still hash-consed); a reversed cycle is a
+    different wiring (transposes) and is not reused."""
+    ctx = _ctx()
+    rng = np.random.default_rng(5)
+    A, B, C, D, E = [ctx.add_node(rng.standard_normal((1, 4, 4)) + 0j) for _ in range(5)]
+    cyc = workloads.meson_cycle_edges
+    ctx.add_graph([A, B, C], cyc(3), [0, 1, 2])
+    s0, _ = ctx.plan(1, [0, 0, 0])
+    ctx.add_graph([B, C, A], cyc(3), [2, 0, 1])          # rotation
+    ctx.add_graph([C, A, B], cyc(3), None)               # rotation, greedy order
+    s1, _ = ctx.plan(1, [0, 0, 0])
+    assert s1["component_dedup_hits"] == 2 and s1["unique_tasks"] == s0["unique_tasks"]
+    two = [(0, 1, 1, 0), (1, 1, 0, 0), (2, 1, 3, 0), (3, 1, 2, 0)]  # tr(XY)·tr(ZW)
+    ctx.add_graph([A, D, B, E], two, None)
+    s2, _ = ctx.plan(1, [0, 0, 0])
+    ctx.add_graph([B, E, A, D], two, None)               # the two components swapped
+    s3, _ = ctx.plan(1, [0, 0, 0])
+    assert s3["component_dedup_hits"] == s2["component_dedup_hits"] + 2
+    assert s3["unique_tasks"] == s2["unique_tasks"]
+    ctx.add_graph([A, D, C, E], two, None)               # tr(AD) known, tr(CE) new
+    s4, _ = ctx.plan(1, [0, 0, 0])
+    assert s4["component_dedup_hits"] == s3["component_dedup_hits"] and s4["unique_tasks"] == s3["unique_tasks"] + 1
+    rev = [(0, 0, 1, 1), (1, 0, 2, 1), (2, 0, 0, 1)]      # tr(A^T B^T C^T)-style reversed wiring
+    ctx.add_graph([A, B, C], rev, None)
+    s5, _ = ctx.plan(1, [0, 0, 0])
+    assert s5["component_dedup_hits"] == s4["component_dedup_hits"]
