@@ -128,14 +128,20 @@ void build_graph(Context &ctx, int32_t n_inst, const int64_t *node_ids, int32_t 
   {
     std::vector<int32_t> parent(n_inst);
     std::iota(parent.begin(), parent.end(), 0);
-    std::function<int32_t(int32_t)> find = [&](int32_t x) { return parent[x] == x ? x : parent[x] = find(parent[x]); };
+    auto find = [&](int32_t x) {  // iterative, path halving (graphs may have 2^20 instances)
+      while (parent[x] != x) x = parent[x] = parent[parent[x]];
+      return x;
+    };
     for (int e = 0; e < n_edges; ++e) parent[find(edges[e].u)] = find(edges[e].v);
     for (int u = 0; u < n_inst; ++u) comp_root[u] = find(u);
   }
+  // members and edges of each component, bucketed once
+  std::vector<std::vector<int32_t>> comp_members(n_inst), comp_edges(n_inst);
+  for (int u = 0; u < n_inst; ++u) comp_members[comp_root[u]].push_back(u);
+  for (int e = 0; e < n_edges; ++e) comp_edges[comp_root[edges[e].u]].push_back(e);
+  std::vector<int32_t> pos(n_inst, -1);
   auto component_key = [&](int32_t root) -> std::string {
-    std::vector<int32_t> mem;
-    for (int u = 0; u < n_inst; ++u)
-      if (comp_root[u] == root) mem.push_back(u);
+    std::vector<int32_t> mem = comp_members[root];
     std::stable_sort(mem.begin(), mem.end(), [&](int32_t x, int32_t y) { return node_ids[x] < node_ids[y]; });
     // tie groups (equal node ids) are permuted among themselves
     std::vector<std::pair<int, int>> groups;
@@ -149,24 +155,23 @@ void build_graph(Context &ctx, int32_t n_inst, const int64_t *node_ids, int32_t 
     }
     if (orders > 5040) return std::string();
     std::vector<int64_t> best;
-    std::vector<int32_t> pos(n_inst, -1);
     std::vector<int32_t> cur = mem;
+    std::vector<std::pair<int64_t, int64_t>> ek;
     std::function<void(size_t)> rec = [&](size_t gi) {
       if (gi == groups.size()) {
         for (size_t i = 0; i < cur.size(); ++i) pos[cur[i]] = (int32_t)i;
         std::vector<int64_t> key;
         key.push_back((int64_t)cur.size());
         for (int32_t u : cur) key.push_back(node_ids[u]);
-        std::vector<int64_t> ek;
-        for (int e = 0; e < n_edges; ++e) {
+        ek.clear();
+        for (int32_t e : comp_edges[root]) {
           const micco_edge &E = edges[e];
-          if (comp_root[E.u] != root) continue;
           int64_t a = (int64_t)pos[E.u] * 8 + E.p, b = (int64_t)pos[E.v] * 8 + E.q;
           if (a > b) std::swap(a, b);
-          ek.push_back(a * 4096 + b);
+          ek.push_back({a, b});
         }
         std::sort(ek.begin(), ek.end());
-        key.insert(key.end(), ek.begin(), ek.end());
+        for (const auto &ab : ek) { key.push_back(ab.first); key.push_back(ab.second); }
         if (best.empty() || key < best) best.swap(key);
         return;
       }
@@ -182,6 +187,8 @@ void build_graph(Context &ctx, int32_t n_inst, const int64_t *node_ids, int32_t 
   for (int u = 0; u < n_inst; ++u)
     if (comp_root[u] == u) roots.push_back(u);
   std::vector<std::string> keys(roots.size());
+  std::vector<int32_t> key_of_root(n_inst, -1);
+  for (size_t i = 0; i < roots.size(); ++i) key_of_root[roots[i]] = (int32_t)i;
   {
     bool all_known = true;
     for (size_t i = 0; i < roots.size(); ++i) {
@@ -473,9 +480,8 @@ void build_graph(Context &ctx, int32_t n_inst, const int64_t *node_ids, int32_t 
         if (comps[u].alive) {
           ctx.graph_scalars.push_back(comps[u].tensor);
           // record the component for canonical reuse (its members share comp_root)
-          for (size_t i = 0; i < roots.size(); ++i)
-            if (comp_root[u] == roots[i] && !keys[i].empty())
-              ctx.component_by_key.emplace(keys[i], std::make_pair(comps[u].tensor, comps[u].flops));
+          const std::string &k = keys[key_of_root[comp_root[u]]];
+          if (!k.empty()) ctx.component_by_key.emplace(k, std::make_pair(comps[u].tensor, comps[u].flops));
         }
       g.comp_end = (int32_t)ctx.graph_scalars.size();
       g.flops_no_dedup = flops_nd;

@@ -390,3 +390,39 @@ def test_canonical_component_reuse():
     ctx.add_graph([A, B, C], rev, None)
     s5, _ = ctx.plan(1, [0, 0, 0])
     assert s5["component_dedup_hits"] == s4["component_dedup_hits"]
+
+
+def test_canonical_component_reuse_large_component():
+    """A 600-instance trace (edge keys past the 4096-leg range of a packed encoding) and 300
+    disjoint two-meson traces: a rotation of the long trace and a reshuffle of the short ones
+    are reused whole; a long trace with two neighbours swapped is a different wiring."""
+    ctx = _ctx()
+    rng = np.random.default_rng(9)
+    ids = [ctx.add_node(rng.standard_normal((1, 2, 2)) + 0j) for _ in range(600)]
+    cyc = workloads.meson_cycle_edges
+    ctx.add_graph(ids, cyc(600), None)
+    s0, _ = ctx.plan(1, [0, 0, 0])
+    ctx.add_graph(ids[217:] + ids[:217], cyc(600), None)
+    s1, _ = ctx.plan(1, [0, 0, 0])
+    assert s1["component_dedup_hits"] == s0["component_dedup_hits"] + 1
+    assert s1["unique_tasks"] == s0["unique_tasks"]
+    sw = list(ids)
+    sw[300], sw[301] = sw[301], sw[300]
+    ctx.add_graph(sw, cyc(600), None)
+    s2, _ = ctx.plan(1, [0, 0, 0])
+    assert s2["component_dedup_hits"] == s1["component_dedup_hits"]
+    pairs = [(0, 1, 1, 0), (1, 1, 0, 0)]
+    inst, edges = [], []
+    for i in range(300):
+        inst += [ids[2 * i], ids[2 * i + 1]]
+        edges += [(a + 2 * i, la, b + 2 * i, lb) for (a, la, b, lb) in pairs]
+    ctx.add_graph(inst, edges, None)
+    s3, _ = ctx.plan(1, [0, 0, 0])
+    perm = rng.permutation(300)
+    inst2 = []
+    for i in perm:
+        inst2 += [ids[2 * i + 1], ids[2 * i]]
+    ctx.add_graph(inst2, edges, None)
+    s4, _ = ctx.plan(1, [0, 0, 0])
+    assert s4["component_dedup_hits"] == s3["component_dedup_hits"] + 300
+    assert s4["unique_tasks"] == s3["unique_tasks"]
