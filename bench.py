@@ -311,7 +311,7 @@ def run_block(M, torch, ctx, wl, world, n_exec, steps, warmup, e2e_steps, dist, 
 def gemm_roofline(b, traffic, traffic_note):
     g = b["gemm"]
     burst, sustained = g["peak"]
-    return {"bound": "tensor", "kernel": "zgemm_persistent (3M, grouped per layout class)",
+    return {"bound": "tensor", "kernel": "zgemm_tma (TMA warp-specialized, meson GEMMs with M >= 128) + zgemm_persistent (cp.async, the other layouts); 3M, grouped per layout class",
             "achieved": g["achieved"], "peak": sustained, "unit": "TFLOP/s", "frac": g["achieved"] / sustained,
             "peak_source": "FP64 DMMA ceiling measured live in this run (micco_probe_fp64_peak: register-only "
                            "mma.sync m8n8k4 f64 loop, back to back, sustained); MEASURED_PEAKS.json has no FP64 entry",
