@@ -470,6 +470,12 @@ def main():
     pc = None
     if n_exec > 1 and not args.no_policy_compare:
         pc = policy_compare(M, torch, args, world, n_exec, dist, local_rank, peak)
+    elif world == 1 and not args.no_policy_compare:
+        # one GPU: the comparison on two logical GPUs of this device (the scheduler, cache and
+        # peer-move paths run; a peer move is a device-local copy here, not NVLink)
+        pc = policy_compare(M, torch, args, 1, 2, None, local_rank, peak)
+        pc["note"] = ("2 logical GPUs on one B200 (micco_execute n_gpus=2 in one process): peer moves are "
+                      "device-local copies, so peer-byte differences weigh less than over NVLink")
 
     if rank != 0:
         if dist is not None:
