@@ -17,6 +17,7 @@
 #include <cuda_runtime.h>
 #include <dlfcn.h>
 #include <nccl.h>
+#include <nvtx3/nvToolsExt.h>  // header-only NVTX v3: no cost unless a profiler injects itself
 
 #include <algorithm>
 #include <array>
@@ -41,6 +42,15 @@ namespace micco {
     if (e_ != cudaSuccess)                                                                          \
       fail(MICCO_ERR_CUDA, std::string("CUDA error: ") + cudaGetErrorString(e_) + " at " #x);       \
   } while (0)
+
+// NVTX ranges (SURVEY.md §5 tracing): execute, planning, each flushed chunk of a stage, host
+// and peer copies, so an nsys / ncu timeline shows the host-side structure of a step.
+struct NvtxRange {
+  explicit NvtxRange(const char *name) { nvtxRangePushA(name); }
+  ~NvtxRange() { nvtxRangePop(); }
+  NvtxRange(const NvtxRange &) = delete;
+  NvtxRange &operator=(const NvtxRange &) = delete;
+};
 
 // ------------------------------------------------------------------ NCCL (dlopen)
 
@@ -484,6 +494,7 @@ struct Executor::Impl {
   }
 
   void flush(LGpu &l) {
+    NvtxRange nr("micco flush");
     CK(cudaSetDevice(l.dev));
     if (!l.gemm.empty()) {  // one grouped launch per operand-layout class
       std::vector<GemmDesc> by[kGemmClasses];
@@ -649,6 +660,7 @@ struct Executor::Impl {
   void run_op(const PlanOp &op, micco_stats &st) {
     switch (op.kind) {
       case PlanOp::H2D: {
+        NvtxRange nr("micco h2d");
         // Prefetch on the copy stream (NEXT #1 of SURVEY.md §8(f); "asynchronous
         // data copy and prefetching"): the copy for chunk k+1 may start once chunk k-1 has
         // finished (bounded look-ahead: at most prefetch_cap bytes beyond the planned budget);
@@ -691,6 +703,7 @@ struct Executor::Impl {
         return;
       }
       case PlanOp::P2P: {  // on the peer stream, ordered with the kernels by events (pace_peer)
+        NvtxRange nr("micco p2p");
         LGpu &dst = g[op.gpu];
         LGpu &src = g[op.src];
         const int64_t nb = bytes_of(op.id);
@@ -817,6 +830,7 @@ struct Executor::Impl {
   }
 
   void execute_impl(int n_gpus, const int32_t *bd) {
+    NvtxRange nr("micco_execute");
     auto t0 = std::chrono::steady_clock::now();
     setup(n_gpus);
     for (auto &l : g)
@@ -896,6 +910,7 @@ struct Executor::Impl {
     if (streaming) {
       in.stream = &ps;
       planner = std::thread([&] {
+        NvtxRange pr("micco plan (streamed)");
         auto p0 = std::chrono::steady_clock::now();
         try {
           plan = make_plan(c, in);
@@ -907,6 +922,7 @@ struct Executor::Impl {
         ps.finish();
       });
     } else {
+      NvtxRange pr(sweep ? "micco plan (bound sweep)" : "micco plan");
       if (sweep) {
         plan = make_plan_auto(c, in);
         for (int i = 0; i < 3; ++i) chosen_bd[i] = plan.reuse_bound[i];

@@ -212,7 +212,6 @@ struct PCfg {
   static constexpr int AE = TBM * APITCH2, BE = BK2 * BP;
   static constexpr int SMEM = ST2 * (AE + BE) * 16;
 };
-constexpr int GEMM2_SMEM = PCfg<64, 64>::SMEM;
 
 // Per-thread load geometry of one operand stage, compile-time for a layout class.  A stage
 // holds ROWS × BK2 complex elements (rows = m for A, n for B); KFAST = the operand is
