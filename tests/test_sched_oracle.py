@@ -73,3 +73,28 @@ def test_eviction_mode_prefers_free_memory():
     assert S.assign(p, [0, 1]) == 1
     S.mem = [10, 10]
     assert S.assign(p, [0, 1]) == 0   # no oversubscription: least computation
+
+
+def test_alg2_tie_breaks():
+    """Alg. 2's ties: with no oversubscription, lines 7-10 take the least
+    computation and, when several GPUs tie on it (GPUSelect.size() > 1), the least memory among
+    them; under oversubscription, lines 12-16 take the least memory (the most capacity, Step-III
+    L250) and break ties on it by the least computation.  Remaining ties go to the lowest id
+    (reading #17 for the paper's random())."""
+    S = MiccoSchedulerOracle(3, [0, 0, 0], gpu_max_memory=1000)
+    S.begin_vector(3)
+    p = Pair(1, 2, 3, 1.0, 5, 5, 5)
+    S.com = [2.0, 2.0, 2.0]
+    S.mem = [30, 10, 20]
+    assert S.assign(p, [0, 1, 2]) == 1          # computation tied: least memory
+    S.com = [2.0, 1.0, 2.0]
+    assert S.assign(p, [0, 1, 2]) == 1          # least computation first
+    S.com = [3.0, 3.0, 1.0]
+    S.mem = [10, 10, 40]
+    assert S.assign(p, [0, 1]) == 0             # full tie: lowest id
+    # oversubscribed (GPU 2 would exceed the budget): least memory, ties by least computation
+    S.mem = [50, 50, 990]
+    S.com = [4.0, 1.0, 0.0]
+    assert S.assign(p, [0, 1, 2]) == 1
+    S.com = [1.0, 4.0, 0.0]
+    assert S.assign(p, [0, 1, 2]) == 0
