@@ -295,7 +295,8 @@ def run_block(M, torch, ctx, wl, world, n_exec, steps, warmup, e2e_steps, dist, 
                          "peak_source": hbm_src, "launches": int(sum(s["dot_main_launches"] for s in stats)),
                          "share_of_step": dot_ms / sum(step_ms),
                          "achieved_note": "algorithmic bytes (16 B per element of both operands, all slices) / "
-                                          "dot launch time (CUDA events on the launching stream)",
+                                          "dot device time (CUDA events on the launching stream, union of "
+                                          "the launches' intervals)",
                          "traffic": None},
         "e2e": ({"value": G / (statistics.mean(e2e_ms) / 1e3), "unit": "graphs/s",
                  "h2d_bytes_per_step": int(statistics.mean(e2e_h2d)), "d2h_bytes_per_step": int(wl.Lt * 16),
@@ -318,8 +319,10 @@ def gemm_roofline(b, traffic, traffic_note):
             "peak_burst": burst, "traffic": traffic, "traffic_note": traffic_note,
             "gemm_launches": g["launches"], "complex_scheme": "3M (3 DMMA products per complex MAC)",
             "executed_dmma_tflops": g["executed"], "executed_frac": g["executed"] / sustained,
-            "achieved_note": "algorithmic ZGEMM-convention flops (8 per complex MAC, SURVEY §8(d)) / GEMM launch "
-                             "time (CUDA events on the launching stream); 3M issues 3/4 of them to the DMMA pipe",
+            "achieved_note": "algorithmic ZGEMM-convention flops (8 per complex MAC, SURVEY §8(d)) / GEMM device "
+                             "time (CUDA events on the launching streams; the union of the launches' intervals, "
+                             "since a chunk's launches alternate between two streams); 3M issues 3/4 of them to "
+                             "the DMMA pipe",
             "gemm_share_of_step": g["share"]}
 
 

@@ -190,8 +190,9 @@ typedef struct {
   size_t struct_size;
   double wall_ms;              /* micco_execute wall time */
   double sched_ms;             /* planning + scheduling (host) */
-  double kernel_ms;            /* device time inside contraction kernels (CUDA events) */
-  double copy_ms;              /* device time of H2D / P2P / D2H copies */
+  double kernel_ms;            /* device time inside contraction kernels (CUDA events; the union
+                                  of the launches' intervals per device, summed over devices) */
+  double copy_ms;              /* device time of the timed H2D copies (same union rule) */
   int64_t bytes_h2d, bytes_p2p, bytes_d2h;
   int64_t evictions;           /* replicas dropped or spilled to make room */
   int64_t cache_hits;          /* operand uses served by a resident replica */
@@ -206,7 +207,8 @@ typedef struct {
   int32_t reuse_bound[3];      /* bounds used (after auto-selection) */
   int32_t n_gpus;
   double gemm_kernel_ms;       /* device time of the GEMM launches only (CUDA events on the
-                                  launching stream, summed over launches) */
+                                  launching stream; union of their intervals: a chunk's launches
+                                  overlap on two streams) */
   double dot_kernel_ms;        /* device time of the dot/trace launches only */
   int64_t gemm_launches, dot_launches;
   double gemm_flops;           /* algorithmic flops of the GEMM-shaped tasks executed */

@@ -162,6 +162,12 @@ struct LGpu {
   cudaStream_t st = nullptr;   // compute stream: kernels, P2P, spills, frees
   cudaStream_t cst = nullptr;  // copy stream: H2D prefetch (async, overlaps the kernels)
   cudaStream_t pst = nullptr;  // peer stream: NVLink moves (peer copies / NCCL send-recv)
+  // side stream of a flushed chunk (forked from st, joined back into it): the chunk's GEMM
+  // launches alternate between st and kst[0], so one persistent launch's last, partly empty
+  // wave overlaps the next launch's first (a chunk's tasks are independent).  The dots stay on
+  // st after the join: run beside the GEMMs they only stretched the GEMM launches (C3: same
+  // step time, 42.8 → 39.6 TF/s of GEMM device time).
+  cudaStream_t kst[1] = {nullptr};
   std::vector<cudaEvent_t> flush_ev;  // compute-stream event after each flushed chunk
   std::vector<int64_t> chunk_fetch;   // bytes fetched for each flushed chunk
   std::vector<int64_t> fetch_bytes_since;
@@ -188,6 +194,7 @@ struct Executor::Impl {
   std::vector<DevState> devs;
   std::vector<ScalarTable> tables;  // indexed by table_of(logical GPU)
   std::vector<Timed> timed;
+  std::vector<cudaEvent_t> time_ref;  // per device: origin of the timed intervals
   std::unordered_map<int32_t, double *> spill_host;
   std::unordered_map<int32_t, std::pair<int, cudaEvent_t>> spill_ev;
   HostArena spill_arena;
@@ -212,6 +219,7 @@ struct Executor::Impl {
   int vals_dev = 0;
   double2 *h_corr = nullptr;
   int64_t launches = 0, tma_launches = 0, oom_retries = 0;
+  int launch_seq = 0;  // launches of the chunk being flushed (side-stream choice)
   bool use_tma = true;  // TMA GEMM for the contractions that fit it (see execute)
   bool dist() const { return c.opt.dist_world > 0; }
   int table_of(int i) const { return c.opt.scalar_tables ? i : g[i].dev; }
@@ -260,11 +268,17 @@ struct Executor::Impl {
     cudaStreamSynchronize(l.st);
     if (l.cst) cudaStreamSynchronize(l.cst);
     if (l.pst) cudaStreamSynchronize(l.pst);
+    for (cudaStream_t k : l.kst)
+      if (k) cudaStreamSynchronize(k);
     l.readers.clear();
     if (destroy_stream) {
       cudaStreamDestroy(l.st);
       cudaStreamDestroy(l.cst);
       cudaStreamDestroy(l.pst);
+      for (cudaStream_t &k : l.kst) {
+        if (k) cudaStreamDestroy(k);
+        k = nullptr;
+      }
       l.pst = nullptr;
       l.st = nullptr;
       l.cst = nullptr;
@@ -318,6 +332,7 @@ struct Executor::Impl {
       CK(cudaStreamCreateWithFlags(&l.st, cudaStreamNonBlocking));
       CK(cudaStreamCreateWithFlags(&l.cst, cudaStreamNonBlocking));
       CK(cudaStreamCreateWithFlags(&l.pst, cudaStreamNonBlocking));
+      for (cudaStream_t &k : l.kst) CK(cudaStreamCreateWithFlags(&k, cudaStreamNonBlocking));
     }
     // Peer access to stream-ordered pool memory is granted per pool (cudaDeviceEnablePeerAccess
     // covers cudaMalloc memory only): every device in use may read every other's pool, so a
@@ -475,27 +490,39 @@ struct Executor::Impl {
   }
 
   template <typename D, typename Batch, typename Prefix>
-  void launch_batch(LGpu &l, std::vector<D> &v, int kind, int cls, Batch &b, int cap, Prefix &&prefix) {
+  void launch_batch(LGpu &l, std::vector<D> &v, int kind, int cls, Batch &b, int cap, Prefix &&prefix,
+                    cudaStream_t (*pick)(LGpu &, int) = nullptr) {
     if (v.empty()) return;
     for (size_t i0 = 0; i0 < v.size(); i0 += (size_t)cap) {
       const int cnt = (int)std::min((size_t)cap, v.size() - i0);
       b.n = cnt;
       std::memcpy(b.d, &v[i0], cnt * sizeof(D));
       const long long total = prefix(b.d, cnt);  // grid offsets of this launch
+      const cudaStream_t s = pick ? pick(l, launch_seq++) : l.st;
       Timed tm{devs[l.dev].timing_events.get(), devs[l.dev].timing_events.get(), kind, l.dev};
-      CK(cudaEventRecord(tm.a, l.st));
-      if constexpr (std::is_same<D, GemmDesc>::value) CK(launch_gemm_group(&b, total, cls, l.st));
-      else CK(launch_dot_group(&b, total, cls, l.st));
-      CK(cudaEventRecord(tm.b, l.st));
+      CK(cudaEventRecord(tm.a, s));
+      if constexpr (std::is_same<D, GemmDesc>::value) CK(launch_gemm_group(&b, total, cls, s));
+      else CK(launch_dot_group(&b, total, cls, s));
+      CK(cudaEventRecord(tm.b, s));
       timed.push_back(tm);
       ++launches;
     }
     v.clear();
   }
 
+  static cudaStream_t pick_gemm(LGpu &l, int seq) { return (seq & 1) ? l.kst[0] : l.st; }
+
   void flush(LGpu &l) {
     NvtxRange nr("micco flush");
     CK(cudaSetDevice(l.dev));
+    if (l.gemm.empty() && l.dot.empty()) return;
+    // fork the side stream off the compute stream (after this chunk's allocations and copy
+    // waits) when the chunk has more than one GEMM launch; joined back below, before the dots
+    launch_seq = 0;
+    if (!l.gemm.empty()) {
+      const cudaEvent_t fork = record_on(l.idx, l.st);
+      for (cudaStream_t k : l.kst) CK(cudaStreamWaitEvent(k, fork, 0));
+    }
     if (!l.gemm.empty()) {  // one grouped launch per operand-layout class
       std::vector<GemmDesc> by[kGemmClasses];
       std::vector<size_t> tma_idx[kGemmClasses];
@@ -518,10 +545,11 @@ struct Executor::Impl {
             b.d[k].tile_begin = acc;
             acc += (long long)b.d[k].Lt * b.d[k].Mo * b.d[k].No * b.d[k].tilesM * b.d[k].tilesN;
           }
+          const cudaStream_t s = pick_gemm(l, launch_seq++);
           Timed tm{devs[l.dev].timing_events.get(), devs[l.dev].timing_events.get(), 0, l.dev};
-          CK(cudaEventRecord(tm.a, l.st));
-          CK(launch_gemm_tma_group(&b, acc, c, l.st));
-          CK(cudaEventRecord(tm.b, l.st));
+          CK(cudaEventRecord(tm.a, s));
+          CK(launch_gemm_tma_group(&b, acc, c, s));
+          CK(cudaEventRecord(tm.b, s));
           timed.push_back(tm);
           ++launches;
           ++tma_launches;
@@ -537,8 +565,10 @@ struct Executor::Impl {
             acc += (long long)d[i].Lt * d[i].Mo * d[i].No * d[i].tilesM * d[i].tilesN;
           }
           return acc;
-        });
+        }, pick_gemm);
     }
+    if (launch_seq > 1)  // join (with one launch the side stream got no work)
+      for (cudaStream_t k : l.kst) CK(cudaStreamWaitEvent(l.st, record_on(l.idx, k), 0));
     if (!l.dot.empty()) {  // one launch group per dot kernel (kernels.h dot_class)
       std::vector<DotDesc> by[2];
       for (const DotDesc &d : l.dot) by[dot_class(d.mode)].push_back(d);
@@ -808,6 +838,8 @@ struct Executor::Impl {
       cudaStreamSynchronize(l.st);
       if (l.cst) cudaStreamSynchronize(l.cst);
       if (l.pst) cudaStreamSynchronize(l.pst);
+      for (cudaStream_t k : l.kst)
+        if (k) cudaStreamSynchronize(k);
       for (auto &p : l.ptr)
         if (p) { cudaFree(p); p = nullptr; }
       for (double2 *p : l.part_allocs) cudaFree(p);
@@ -846,6 +878,15 @@ struct Executor::Impl {
       l.pending_fetch = 0;
     }
     for (auto &d : devs) { d.sync_events.reset(); d.timing_events.reset(); }
+    // per-device time origin of the kernel/copy intervals (the streams are idle here, so every
+    // later launch on any stream of the device starts after it)
+    time_ref.assign(ndev, nullptr);
+    for (auto &l : g)
+      if (l.local && !time_ref[l.dev]) {
+        time_ref[l.dev] = devs[l.dev].timing_events.get();
+        CK(cudaSetDevice(l.dev));
+        CK(cudaEventRecord(time_ref[l.dev], l.st));
+      }
 
     PlanInput in;
     in.n_gpus = n;
@@ -1097,20 +1138,42 @@ struct Executor::Impl {
     spill_ev.clear();
     spill_arena.rewind();  // keep the pinned spill chunks for the next execute
 
-    // statistics
-    for (const Timed &tm : timed) {
-      float ms = 0;
-      CK(cudaSetDevice(tm.dev));
-      CK(cudaEventElapsedTime(&ms, tm.a, tm.b));
-      if (tm.kind == 2) { st.copy_ms += ms; continue; }
-      st.kernel_ms += ms;
-      if (tm.kind == 0) { st.gemm_kernel_ms += ms; ++st.gemm_launches; }
-      else if (tm.kind == 1) { st.dot_kernel_ms += ms; ++st.dot_launches; }
-      else if (tm.kind == 3) {
-        st.dot_kernel_ms += ms;
-        ++st.dot_launches;
-        st.dot_main_ms += ms;
-        ++st.dot_main_launches;
+    // statistics: device time per kind = the union of its launches' intervals on each device
+    // (launches of one chunk overlap on the side streams, so a plain sum would count the
+    // overlap twice), summed over devices
+    {
+      std::vector<std::pair<float, float>> iv[5];  // gemm, dot (warp), copy, dot (CTA), all kernels
+      auto union_ms = [](std::vector<std::pair<float, float>> &v) {
+        std::sort(v.begin(), v.end());
+        double tot = 0, a = 0, b = -1;
+        for (const auto &x : v) {
+          if (x.first > b) { if (b > a) tot += b - a; a = x.first; b = x.second; }
+          else b = std::max(b, (double)x.second);
+        }
+        if (b > a) tot += b - a;
+        v.clear();
+        return tot;
+      };
+      for (int d = 0; d < ndev; ++d) {
+        if (d >= (int)time_ref.size() || !time_ref[d]) continue;
+        CK(cudaSetDevice(d));
+        for (const Timed &tm : timed) {
+          if (tm.dev != d) continue;
+          float a = 0, b = 0;
+          CK(cudaEventElapsedTime(&a, time_ref[d], tm.a));
+          CK(cudaEventElapsedTime(&b, time_ref[d], tm.b));
+          iv[tm.kind].push_back({a, b});
+          if (tm.kind != 2) iv[4].push_back({a, b});
+          if (tm.kind == 0) ++st.gemm_launches;
+          else if (tm.kind == 1) ++st.dot_launches;
+          else if (tm.kind == 3) { ++st.dot_launches; ++st.dot_main_launches; }
+        }
+        st.gemm_kernel_ms += union_ms(iv[0]);
+        st.copy_ms += union_ms(iv[2]);
+        iv[1].insert(iv[1].end(), iv[3].begin(), iv[3].end());
+        st.dot_main_ms += union_ms(iv[3]);
+        st.dot_kernel_ms += union_ms(iv[1]);
+        st.kernel_ms += union_ms(iv[4]);
       }
     }
     st.wall_ms = std::chrono::duration<double, std::milli>(t2 - t0).count();
