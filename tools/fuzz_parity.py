@@ -116,13 +116,21 @@ def main():
             evictions += st["evictions"]
             p2p += st["bytes_p2p"]
             for C, vals in res:
-                if wl.mode == MODE_INT3:
-                    ok = np.array_equal(vals, valso) and np.array_equal(C, Co)
+                if wl.mode == MODE_INT3:  # graph values exact; C(t) sums random complex c_g (rounded)
+                    ok = np.array_equal(vals, valso) and rel_err(C, Co) <= TOL
                 else:
                     ok = rel_err(C, Co) <= TOL and all(rel_err(vals[g], valso[g]) <= TOL for g in range(len(wl.graphs)))
                 if not ok:
-                    print(json.dumps({"FAIL": wl.name, "case": case, "opts": opts, "n": n, "bd": bd,
-                                      "err": rel_err(C, Co)}), flush=True)
+                    errs = [rel_err(vals[g], valso[g]) for g in range(len(wl.graphs))]
+                    bad = [g for g in range(len(wl.graphs)) if not (errs[g] <= TOL) or
+                           (wl.mode == MODE_INT3 and not np.array_equal(vals[g], valso[g]))]
+                    print(json.dumps({"FAIL": wl.name, "case": case, "mode": wl.mode, "Lt": wl.Lt, "opts": opts,
+                                      "n": n, "bd": bd, "err_C": rel_err(C, Co), "bad_graphs": bad[:10],
+                                      "errs": [errs[g] for g in bad[:10]],
+                                      "graphs": [(wl.graphs[g].inst, wl.graphs[g].edges, wl.graphs[g].order)
+                                                 for g in bad[:3]],
+                                      "got": [[str(x) for x in vals[g][:2]] for g in bad[:3]],
+                                      "want": [[str(x) for x in valso[g][:2]] for g in bad[:3]]}), flush=True)
                     sys.exit(1)
                 key = bool(opts["reorder"])
                 if key not in ref:
