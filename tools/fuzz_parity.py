@@ -60,6 +60,27 @@ def draw_workload(rng, case):
     return Workload(f"mesons{N}", Lt, case, mode, nodes, graphs)
 
 
+def add_relabeled(rng, wl):
+    """Append copies of random graphs with their instances relabeled (permuted), edges mapped and
+    flipped end for end, and a fresh random order: the canonical component keys must match them
+    to the originals (builder.cpp), and the oracle recomputes them from scratch."""
+    extra = []
+    for _ in range(int(rng.integers(1, 1 + len(wl.graphs)))):
+        g = wl.graphs[int(rng.integers(len(wl.graphs)))]
+        n = len(g.inst)
+        perm = [int(x) for x in rng.permutation(n)]  # old instance u -> new index perm[u]
+        inst = [0] * n
+        for u in range(n):
+            inst[perm[u]] = g.inst[u]
+        edges = []
+        for (u, p_, v, q) in g.edges:
+            e = (perm[u], p_, perm[v], q)
+            edges.append(e if rng.random() < 0.5 else (e[2], e[3], e[0], e[1]))
+        order = [int(x) for x in rng.permutation(len(edges))]
+        extra.append(GraphSpec(inst, edges, order, complex(rng.normal(), rng.normal())))
+    return Workload(wl.name + "+relabeled", wl.Lt, wl.seed, wl.mode, wl.nodes, list(wl.graphs) + extra, wl.meta)
+
+
 def draw_options(rng, wl):
     node_bytes = max(16 * wl.Lt * nd.N ** nd.rank for nd in wl.nodes)
     opts = {"policy": str(rng.choice(POLICIES)), "reorder": bool(rng.random() < 0.5)}
@@ -102,6 +123,8 @@ def main():
         if time.time() - t0 > a.minutes * 60:
             break
         wl = draw_workload(rng, case)
+        if rng.random() < 0.5:
+            wl = add_relabeled(rng, wl)
         Co, valso = oracle.correlator(wl, return_values=True)
         ref = {}  # per reduction order (reorder changes the contraction trees, hence rounding)
         for _ in range(int(rng.integers(1, 4))):
