@@ -1,6 +1,6 @@
 """Localise nondeterministic results: run a workload in fresh contexts, compare every graph value
 val_g(t) with the first run bit for bit, report which (graph, slice) differ and how.
-    python tools/race_hunt.py <c3_10k|c3_2k|c5full> <runs> [executes_per_ctx]"""
+    python tools/race_hunt.py <c3_10k|c3_2k|c4|c5full> <runs> [executes_per_ctx]"""
 import collections
 import sys
 from pathlib import Path
@@ -16,6 +16,8 @@ if cfg == "c3_10k":
     wl, kw = workloads.c3_multi_meson(n_graphs=10000, N=256, Lt=128), dict(reorder=True)
 elif cfg == "c3_2k":
     wl, kw = workloads.c3_multi_meson(n_graphs=2000, N=256, Lt=128), dict(reorder=True)
+elif cfg == "c4":
+    wl, kw = workloads.c4_two_baryon(), {}
 else:
     wl, kw = workloads.c5_mixed(n_combos=4, Nb=64, Nm=256, Lt=64, pool=4, meson_graphs=64), {}
 G, Lt = len(wl.graphs), wl.Lt
