@@ -516,14 +516,12 @@ struct Executor::Impl {
     NvtxRange nr("micco flush");
     CK(cudaSetDevice(l.dev));
     if (l.gemm.empty() && l.dot.empty()) return;
-    // fork the side stream off the compute stream (after this chunk's allocations and copy
-    // waits) when the chunk has more than one GEMM launch; joined back below, before the dots
     launch_seq = 0;
-    if (!l.gemm.empty()) {
+    if (!l.gemm.empty()) {  // one grouped launch per operand-layout class
+      // fork the side stream off the compute stream (after this chunk's allocations and copy
+      // waits); the launches alternate between the two, joined back below before the dots
       const cudaEvent_t fork = record_on(l.idx, l.st);
       for (cudaStream_t k : l.kst) CK(cudaStreamWaitEvent(k, fork, 0));
-    }
-    if (!l.gemm.empty()) {  // one grouped launch per operand-layout class
       std::vector<GemmDesc> by[kGemmClasses];
       std::vector<size_t> tma_idx[kGemmClasses];
       for (size_t i = 0; i < l.gemm.size(); ++i) {
