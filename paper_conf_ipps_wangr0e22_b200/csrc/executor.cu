@@ -27,6 +27,7 @@
 #include <string>
 #include <exception>
 #include <thread>
+#include <tuple>
 #include <type_traits>
 #include <unordered_map>
 
@@ -207,6 +208,7 @@ struct Executor::Impl {
   std::unique_ptr<GemmBatch> gemm_batch{new GemmBatch};  // kernel-parameter staging
   std::unique_ptr<GemmTmaBatch> tma_batch{new GemmTmaBatch};
   std::unique_ptr<DotBatch> dot_batch{new DotBatch};
+  std::unique_ptr<DotGroupBatch> dot_group_batch{new DotGroupBatch};
   int32_t chosen_bd[3] = {0, 0, 0};
   int chosen_bd_n = 0;
   int stream_ok_n = 0;  // GPU count of the last completed execute (its nodes are materialised)
@@ -510,6 +512,38 @@ struct Executor::Impl {
     v.clear();
   }
 
+  // Small dots that share their A operand go to the shared-operand kernel (kernels.h
+  // DotGroupBatch).  Batches keep the plan order (so a launch covers the same operands as an
+  // ungrouped one); inside a batch the descriptors are ordered by A (stable) and consecutive
+  // equal A's form groups of up to kDotGroupPartners (splitting is exact: a dot's value does
+  // not depend on its group).
+  void launch_shared_groups(LGpu &l, std::vector<DotDesc> &v) {
+    auto key = [](const DotDesc &d) {
+      return std::make_tuple((uintptr_t)d.A, d.sAt, d.sAy, d.X, d.Y, d.mode, d.sBt, d.sBx, d.sBy);
+    };
+    DotGroupBatch &b = *dot_group_batch;
+    for (size_t i0 = 0; i0 < v.size(); i0 += kDotGroupBatch) {
+      const int cnt = (int)std::min((size_t)kDotGroupBatch, v.size() - i0);
+      std::stable_sort(v.begin() + i0, v.begin() + i0 + cnt,
+                       [&](const DotDesc &x, const DotDesc &y) { return key(x) < key(y); });
+      b.n = cnt;
+      b.n_groups = 0;
+      for (int k = 0; k < cnt; ++k) {
+        b.d[k] = v[i0 + k];
+        if (k == 0 || key(b.d[k]) != key(b.d[k - 1]) || k - b.first[b.n_groups - 1] == kDotGroupPartners)
+          b.first[b.n_groups++] = (short)k;
+      }
+      b.first[b.n_groups] = (short)cnt;
+      Timed tm{devs[l.dev].timing_events.get(), devs[l.dev].timing_events.get(), 3, l.dev};
+      CK(cudaEventRecord(tm.a, l.st));
+      CK(launch_dot_shared_group(&b, c.Lt, l.st));
+      CK(cudaEventRecord(tm.b, l.st));
+      timed.push_back(tm);
+      ++launches;
+    }
+    v.clear();
+  }
+
   static cudaStream_t pick_gemm(LGpu &l, int seq) { return (seq & 1) ? l.kst[0] : l.st; }
 
   void flush(LGpu &l) {
@@ -568,9 +602,13 @@ struct Executor::Impl {
     if (launch_seq > 1)  // join (with one launch the side stream got no work)
       for (cudaStream_t k : l.kst) CK(cudaStreamWaitEvent(l.st, record_on(l.idx, k), 0));
     if (!l.dot.empty()) {  // one launch group per dot kernel (kernels.h dot_class)
-      std::vector<DotDesc> by[2];
-      for (const DotDesc &d : l.dot) by[dot_class(d.mode)].push_back(d);
+      std::vector<DotDesc> by[2], grp;
+      for (const DotDesc &d : l.dot) {
+        if (dot_class(d.mode) == 1 && dot_groupable(d)) grp.push_back(d);
+        else by[dot_class(d.mode)].push_back(d);
+      }
       l.dot.clear();
+      launch_shared_groups(l, grp);
       for (int c = 0; c < 2; ++c) {
         launch_batch(l, by[c], c == 0 ? 1 : 3, c, *dot_batch, kDotBatch, [](DotDesc *d, int cnt) {
           long long acc = 0;

@@ -1139,6 +1139,72 @@ __device__ __forceinline__ void zdot_body(const DotDesc *__restrict__ descs, int
   }
 }
 
+// Dots of one launch that share their A operand (C4: each c = 2 product is the A side of many
+// final dots), for slices of ≤ kDotGroupElems complex with no outer index: one CTA per (group of
+// ≤ kDotGroupPartners such dots, slice) stages A's slice in shared memory once, in the order its
+// partners are read, and streams the partners B against it, one element of every partner in
+// flight together.  The C4 dot launches were L2-bound (11.6 TB/s served by L2 for 512 MB from
+// DRAM, profiles/r02/ncu_dot_c4_r02.json); staging the shared side cuts their L2 bytes.  Groups
+// are formed inside plan-order batches (a launch covers the same operands as an ungrouped one).
+// Measured on C4 (profiles/r02/dotgroup/): 6 partners at 2 CTAs/SM 49.2 → 43.3 ms of dots per
+// step; 8 partners (larger groups, fewer CTAs) and 2-4 partners at 3 CTAs/SM were slower.
+// Element order, per-thread sums and the reduction tree depend only on the descriptor, never
+// on the group it lands in, so a dot's value is bitwise the same whatever the grouping (GPU
+// counts, windows and batch boundaries change the groups).
+//   term (x, y) = A[y·sAy + x·sAx] · B[x·sBx + y·sBy],  e = x·Y + y enumerates B (sBy = 1 in
+//   mode 1; Y = 1 in mode 0, where x runs contiguous in both)
+// smem S[x·P + y] = A[y][x], P = Y + 1 when Y > 1 (conflict-free transposed staging stores).
+__global__ void __launch_bounds__(DT, 2) zdot_group_kernel(const __grid_constant__ DotGroupBatch b) {
+  extern __shared__ __align__(16) double2 S[];
+  __shared__ double2 red[kDotGroupPartners][DT / 32];
+  const int ng = b.n_groups;
+  const int t = (int)(blockIdx.x / ng), g = (int)(blockIdx.x - (unsigned)t * ng);  // slice-major
+  const int i0 = b.first[g], np = b.first[g + 1] - i0;
+  const DotDesc &d0 = b.d[i0];
+  const int X = d0.X, Y = d0.Y, P = Y > 1 ? Y + 1 : 1, XY = X * Y;
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  {
+    const double2 *A = d0.A + t * d0.sAt;
+    const int sAy = (int)d0.sAy, sAx = (int)d0.sAx;
+#pragma unroll 8
+    for (int e = tid; e < XY; e += DT) {  // coalesced along x (sAx = 1)
+      const int y = e / X, x = e - y * X;
+      S[x * P + y] = ldg_stream(A + y * sAy + x * sAx);
+    }
+  }
+  const double2 *Bp[kDotGroupPartners];  // (a group shares the partners' strides too)
+#pragma unroll
+  for (int p = 0; p < kDotGroupPartners; ++p) Bp[p] = b.d[i0 + (p < np ? p : 0)].B + t * d0.sBt;
+  const int sBx = (int)d0.sBx, sBy = (int)d0.sBy;
+  double sr[kDotGroupPartners], si[kDotGroupPartners];
+#pragma unroll
+  for (int p = 0; p < kDotGroupPartners; ++p) sr[p] = si[p] = 0.0;
+  __syncthreads();
+#pragma unroll 2
+  for (int e = tid; e < XY; e += DT) {  // every partner's element e in flight together
+    const int x = e / Y, y = e - x * Y;
+    const double2 a = S[x * P + y];
+#pragma unroll
+    for (int p = 0; p < kDotGroupPartners; ++p)
+      if (p < np) cmac(sr[p], si[p], a, ldg_stream(Bp[p] + x * sBx + y * sBy));
+  }
+#pragma unroll
+  for (int p = 0; p < kDotGroupPartners; ++p) {
+#pragma unroll
+    for (int off = 16; off > 0; off >>= 1) {
+      sr[p] += __shfl_xor_sync(0xffffffffu, sr[p], off);
+      si[p] += __shfl_xor_sync(0xffffffffu, si[p], off);
+    }
+    if (lane == 0) red[p][warp] = make_double2(sr[p], si[p]);
+  }
+  __syncthreads();
+  if (tid < np) {  // warps in order (the same tree as zdot_body)
+    double ar = 0.0, ai = 0.0;
+    for (int w = 0; w < DT / 32; ++w) { ar += red[tid][w].x; ai += red[tid][w].y; }
+    b.d[i0 + tid].out[t] = make_double2(ar, ai);
+  }
+}
+
 // One warp per (dot, slice) for the short reductions (2: meson trace, 3: sum of the fused
 // GEMM's partials): no block barrier, a fixed-order butterfly (deterministic).  The flat
 // dots (mode 0) stay on the CTA kernel: a warp per C4 64×64 dot put 8× more slices in
@@ -1476,6 +1542,36 @@ cudaError_t launch_dot_group(const DotBatch *b, long long total_ctas, int cls, c
     return cudaGetLastError();
   }
   zdot_kernel<<<(unsigned)total_ctas, DT, 0, st>>>(*b);
+  return cudaGetLastError();
+}
+
+bool dot_groupable(const DotDesc &d) {
+  if (!(d.mode == 0 || d.mode == 1) || !d.B) return false;
+  if (d.O[0] * d.O[1] * d.O[2] != 1 || d.sAx != 1) return false;
+  if ((long long)d.X * d.Y > kDotGroupElems) return false;
+  return d.mode == 0 ? (d.Y == 1 && d.sBx == 1) : d.sBy == 1;
+}
+
+static size_t dot_group_smem(int X, int Y) { return (size_t)X * (Y > 1 ? Y + 1 : 1) * sizeof(double2); }
+
+cudaError_t launch_dot_shared_group(const DotGroupBatch *b, int Lt, cudaStream_t st) {
+  static unsigned long long attr_set = 0;  // per device (see launch_gemm_group)
+  int dev = 0;
+  if (cudaError_t e = cudaGetDevice(&dev); e != cudaSuccess) return e;
+  const unsigned long long bit = 1ull << (dev & 63);
+  if (!(attr_set & bit)) {
+    cudaError_t e = cudaFuncSetAttribute(zdot_group_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         (int)dot_group_smem(64, 64));
+    if (e != cudaSuccess) return e;
+    attr_set |= bit;
+  }
+  if (b->n_groups <= 0 || Lt <= 0) return cudaSuccess;
+  size_t smem = 0;  // the largest group of the batch
+  for (int g = 0; g < b->n_groups; ++g) {
+    const DotDesc &d = b->d[b->first[g]];
+    smem = std::max(smem, dot_group_smem(d.X, d.Y));
+  }
+  zdot_group_kernel<<<(unsigned)((long long)b->n_groups * Lt), DT, smem, st>>>(*b);
   return cudaGetLastError();
 }
 

@@ -110,6 +110,21 @@ cudaError_t launch_gemm_tma_group(const GemmTmaBatch *b, long long total_tiles, 
 inline int dot_class(int mode) { return mode == 0 || mode == 1 ? 1 : 0; }
 cudaError_t launch_dot_group(const DotBatch *b, long long total_ctas, int cls, cudaStream_t st);
 
+// Dots that share their A operand, launched as groups (kernels.cu zdot_group_kernel): the
+// descriptors of a group are consecutive and share A (pointer, strides, extents) and the
+// partners' strides; first[g] is the first descriptor of group g, first[n_groups] = n; a group
+// holds at most kDotGroupPartners descriptors.  Only small slices without outer indices qualify
+// (dot_groupable); the rest stay on launch_dot_group.
+constexpr int kDotGroupBatch = 184, kDotGroupElems = 4096, kDotGroupPartners = 6;
+struct DotGroupBatch {
+  int n, n_groups;
+  short first[kDotGroupBatch + 2];
+  DotDesc d[kDotGroupBatch];
+};
+static_assert(sizeof(DotGroupBatch) <= 32764, "kernel parameter limit");
+bool dot_groupable(const DotDesc &d);
+cudaError_t launch_dot_shared_group(const DotGroupBatch *b, int Lt, cudaStream_t st);
+
 // vals[g][t] = Π_{c in comps(g)} S[slot_c][t] (component scalars)
 cudaError_t launch_finalize(int G, int Lt, const int *comp_off, const int *comp_slot,
                             const double2 *scalars, double2 *vals, cudaStream_t st);

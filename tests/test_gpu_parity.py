@@ -444,6 +444,41 @@ def test_tma_gemm_ragged_tiles():
     assert st["gemm_tma_launches"] > 0, st
 
 
+def test_shared_operand_dot_groups():
+    """The shared-operand dot kernel (kernels.cu zdot_group_kernel): greedy two-baryon graphs at
+    N = 16 (every final dot is a 16 × 16 flat or transposed dot; the c = 2 products are the A side
+    of many dots, so groups fill up to kDotGroupPartners and batches split them), against the
+    oracle, integer inputs bit-exact, and every graph value bitwise the same under other
+    groupings (windows, GPU counts, per-GPU tables); plus meson cycles at N = 64 (the largest
+    groupable slice) and 65 (the CTA dot kernel) against the oracle."""
+    wl = workloads.c4_two_baryon(n_combos=1, N=16, Lt=3, pool=2, order="greedy")
+    C, vals, st = run_gpu(wl)
+    Co, valso = oracle.correlator(wl, return_values=True)
+    assert rel_err(C, Co) <= TOL
+    for g in range(len(wl.graphs)):
+        assert rel_err(vals[g], valso[g]) <= TOL, g
+    for kw in ({"window_graphs": 7}, {"window_graphs": 300}, {"n_gpus": 3, "scalar_tables": 1}):
+        n = kw.pop("n_gpus", 1)
+        C2, vals2, _ = run_gpu(wl, n, **kw)
+        assert np.array_equal(vals2, vals), kw
+        assert np.array_equal(C2, C), kw
+    wli = workloads.c4_two_baryon(n_combos=1, N=16, Lt=2, pool=2, order="greedy", mode=MODE_INT3,
+                                  matchings=list(range(0, 720, 3)))
+    _, vals, _ = run_gpu(wli)
+    _, valso = oracle.correlator(wli, return_values=True)
+    assert np.array_equal(vals, valso)
+    for N in (64, 65):
+        rng = np.random.default_rng(N)
+        nodes = [NodeSpec(2, N, 300 + i) for i in range(3)]
+        graphs = []
+        for k in (2, 2, 3, 4, 4):
+            inst = [int(x) for x in rng.integers(0, 3, size=k)]
+            flips = [bool(x) for x in rng.integers(0, 2, size=k)]
+            graphs.append(GraphSpec(inst, workloads.meson_cycle_edges(k, flips), list(range(k)),
+                                    complex(rng.choice([-1.0, 1.0]))))
+        check(Workload(f"dots{N}", 2, 5 + N, 0, nodes, graphs))
+
+
 def test_repeat_bitwise_at_scale():
     """Bitwise reproducibility of every graph value over repeated executes and fresh contexts at
     C3's tensor size (N = 256, Lt = 128, 2000 graphs, reuse-aware order: TMA GEMMs with fused
